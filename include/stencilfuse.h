@@ -1,0 +1,219 @@
+/*
+ * stencilfuse.h — C ABI of the B200-native stencil-DAG executor.
+ *
+ * The hot path of Wahib & Maruyama, "Automated GPU Kernel Transformations in
+ * Large-Scale Production Stencil Applications" (HPDC'15; /root/reference/PAPER.md,
+ * cited P:L<line> §<section>): a stencil application is a sequence of
+ * memory-bound kernels over shared 3-D arrays (§1, §2); the method
+ * replaces them by fused kernels that keep intermediates on chip with halo
+ * recompute (complex fusion, §5.5.3), input sharing (simple fusion,
+ * P:L288 §5.5.2), after optional fission of kernels into independent pieces
+ * (§4.1, Algorithm 2).  This library executes a program either as
+ * written (run_unfused, "no fusion" P:L284 §5.5.1) or under a fission/fusion
+ * plan (run_fused, host invocation order P:L296 §5.5.4), on one GPU or on a
+ * z-slab decomposition over several GPUs (exchange_halos).
+ *
+ * Conventions
+ *  - Every function returns sp_status; SP_OK == 0.  On error a message is
+ *    available from sp_last_error() (thread-local, valid until the next call
+ *    on the same thread).  No C++ exception crosses this boundary.
+ *  - Host pointers are read during the call only; the library deep-copies
+ *    every description it is given.
+ *  - Device pointers are borrowed (stencil_program_bind): the caller owns the
+ *    memory and keeps it alive while the program may use it.
+ *  - cudaStream_t arguments are borrowed; run_* and exchange_halos are
+ *    asynchronous and stream-ordered.  Launch errors are reported
+ *    synchronously; asynchronous faults surface at the caller's next sync.
+ *  - A handle is not thread-safe; distinct handles are independent.
+ *  - Nothing here falls back to the CPU: without a usable CUDA device the
+ *    device entry points return SP_E_CUDA.
+ */
+#ifndef STENCILFUSE_H
+#define STENCILFUSE_H
+
+#include <stddef.h>
+#include <stdint.h>
+
+#ifdef __cplusplus
+extern "C" {
+#endif
+
+typedef struct CUstream_st *sp_stream; /* == cudaStream_t */
+
+typedef enum {
+    SP_OK = 0,
+    SP_E_ARG = 1,            /* bad argument, size or index                          */
+    SP_E_PROGRAM = 2,        /* program violates the model (R3 race, tap > ghost ...) */
+    SP_E_PLAN_PARTITION = 3, /* a statement missing or listed twice                  */
+    SP_E_PLAN_ORDER = 4,     /* a dependency edge points backwards in the plan       */
+    SP_E_PLAN_HAZARD = 5,    /* a group reads from HBM an array it also stores (R11) */
+    SP_E_RESOURCES = 6,      /* no tile fits shared memory / halo deeper than alloc  */
+    SP_E_JIT = 7,            /* NVRTC compilation or module load failed              */
+    SP_E_CUDA = 8,           /* CUDA runtime/driver error (or no device)             */
+    SP_E_NCCL = 9,           /* NCCL error                                           */
+    SP_E_STATE = 10          /* call not valid in the current state                  */
+} sp_status;
+
+typedef enum { SP_F32 = 4, SP_F64 = 8 } sp_dtype; /* value = element size in bytes */
+
+/* Array roles.  IN: read only.  OUT/INOUT: results compared after a run
+ * (INOUT may also be read first).  TEMP: inter-kernel intermediate whose HBM
+ * content after run_fused is unspecified (reading R6 in DESIGN.md). */
+typedef enum { SP_IN = 1, SP_OUT = 2, SP_INOUT = 3, SP_TEMP = 4 } sp_role;
+
+/* One access a[p + (dx,dy,dz)]; |d| must not exceed the ghost width. */
+typedef struct { int32_t array, dx, dy, dz; } sp_tap;
+
+/* term = coef * a[p+da]            (has_b == 0)
+ *      = (coef * a[p+da]) * b[p+db] (has_b != 0)                       (R4) */
+typedef struct { double coef; sp_tap a; int32_t has_b; sp_tap b; } sp_term;
+
+/* out[p] = term0 + term1 + ... accumulated left to right, for every interior p
+ * (the stencil operations of the paper's "operations metadata", §3.2.1). */
+typedef struct { int32_t out; int32_t n_terms; const sp_term *terms; } sp_stmt;
+
+/* A kernel: ordered statements executed per point (reading R3:
+ * an array written by the kernel may be read by it only at offset 0). */
+typedef struct { const char *name; int32_t n_stmts; const sp_stmt *stmts; } sp_kernel;
+
+typedef struct { const char *name; sp_role role; } sp_array_desc;
+
+/* Grid of THIS process.  z is the marched and the decomposed axis.
+ *   nx, ny      interior size in x (contiguous) and y
+ *   nz_local    interior planes owned by this rank
+ *   nz_global   interior planes of the whole grid (== nz_local on one rank)
+ *   z_offset    global z of local plane 0
+ *   ghost[3]    ghost width per axis (>= max |offset| of any tap)
+ *   zhalo       ghost planes allocated below/above in z (>= ghost[2]); the
+ *               deep halo that fused groups with accumulated z-reach need on
+ *               several ranks.  0 means ghost[2]. */
+typedef struct {
+    int64_t nx, ny, nz_local, nz_global, z_offset;
+    int32_t ghost[3];
+    int32_t zhalo;
+    sp_dtype dtype;
+} sp_grid;
+
+typedef struct { int32_t kernel, stmt; } sp_stmt_ref;
+
+/* Storage of every array (identical for all arrays of a program):
+ * dense [z_alloc][y_alloc][x_pitch] elements, x fastest; interior point
+ * (i,j,k) at ((k+origin_z)*y_alloc + j+origin_y)*x_pitch + i+origin_x.
+ * x_pitch*elem is a multiple of 128 B; base pointers must be 256-B aligned. */
+typedef struct {
+    int64_t x_pitch, y_alloc, z_alloc, origin_x, origin_y, origin_z, bytes;
+} sp_layout;
+
+/* DDG/OEG edge between statements (global statement ids in program order,
+ * P:L104-136 §3.2.3; reading R9/R10).  kind: bit0 RAW, bit1 WAR, bit2 WAW. */
+typedef struct { int32_t from, to, kind, array; } sp_edge;
+
+/* Per-launch report of a group (fused) or kernel (unfused).  Byte/flop figures
+ * are per interior grid point of one launch.                              */
+typedef struct {
+    int32_t n_stmts;          /* statements computed (dead ones excluded)        */
+    int32_t n_inputs;         /* arrays read from HBM (ExtIn)                    */
+    int32_t n_stores;         /* arrays written to HBM (LiveOut, reading R6)      */
+    int32_t n_smem_stages;    /* on-chip stages kept in shared-memory planes      */
+    int32_t n_reg_stages;     /* on-chip stages kept in registers / queues        */
+    int32_t ext[4];           /* max halo extension of any stage: x-, x+, y-, y+  */
+    int32_t z_below, z_above; /* planes read below/above the output plane (reach) */
+    int32_t tile_x, tile_y, zchunk, threads;
+    int32_t grid_ctas;        /* CTAs per launch                                 */
+    int32_t regs_per_thread;  /* after JIT (-1 before)                           */
+    int64_t smem_bytes;       /* dynamic shared memory per CTA                   */
+    double bytes_alg;         /* elem * (|ExtIn| + |LiveOut|)                    */
+    double flops_alg;         /* sum over stmts of 2*terms - 1 + products         */
+    double bytes_exec;        /* incl. halo re-reads and z warm-up planes         */
+    double flops_exec;        /* incl. halo recompute and warm-up                 */
+    double smem_bytes_pt;     /* shared-memory traffic per point (model)          */
+} sp_group_report;
+
+typedef struct sp_comm_s sp_comm;
+typedef struct stencil_program_s stencil_program;
+
+/* ---- communicator (z-slab decomposition) -------------- */
+/* nccl_unique_id: the 128-byte ncclUniqueId produced by rank 0 (sp_comm_unique_id)
+ * and broadcast by the caller (e.g. torch.distributed).  The current CUDA
+ * device of the calling thread is used.  Collective over nranks. */
+sp_status sp_comm_unique_id(void *out128);
+sp_status sp_comm_create(const void *nccl_unique_id, int32_t nranks, int32_t rank, sp_comm **out);
+void sp_comm_destroy(sp_comm *comm);
+
+/* ---- program ------------------------------------------------------------ */
+/* Validates and deep-copies the program (kernels in host invocation order,
+ * P:L136).  comm may be NULL (single rank).  Errors: SP_E_ARG (sizes),
+ * SP_E_PROGRAM (tap beyond ghost, unknown array, R3 in-kernel race,
+ * statement without terms). */
+sp_status stencil_program_create(const sp_grid *grid, int32_t n_arrays, const sp_array_desc *arrays,
+                                 int32_t n_kernels, const sp_kernel *kernels, sp_comm *comm,
+                                 stencil_program **out);
+void stencil_program_destroy(stencil_program *prog);
+
+sp_status stencil_program_layout(const stencil_program *prog, sp_layout *out);
+
+/* Borrow dev_ptr (caller-owned, >= layout.bytes, 256-B aligned) as array `array`. */
+sp_status stencil_program_bind(stencil_program *prog, int32_t array, void *dev_ptr);
+
+/* Tuning/parity options; must precede fusion_plan_set / the first run.
+ *   "fmad"      0|1  FMA contraction in generated code (default 1; 0 = parity build)
+ *   "tile_x", "tile_y", "zchunk", "threads", "prefetch"   override the tile chooser
+ *   "l2_flush"  unused by the library (reserved) */
+sp_status sp_program_set_option(stencil_program *prog, const char *key, int64_t value);
+
+sp_status sp_program_counts(const stencil_program *prog, int32_t *n_stmts, int32_t *n_edges);
+/* Copies up to cap edges (all RAW/WAR/WAW statement pairs in program order). */
+sp_status sp_program_edges(const stencil_program *prog, int32_t cap, sp_edge *out, int32_t *n);
+
+/* Kernel fission (§4.1, Algorithm 2; reading R8): connected
+ * components of the graph joining each statement's output array with every
+ * array it reads.  comp_of_stmt[i] receives the piece of statement i of the
+ * kernel, pieces numbered in order of their first statement.  */
+sp_status sp_fission_components(const stencil_program *prog, int32_t kernel, int32_t *comp_of_stmt,
+                                int32_t *n_comp);
+
+/* ---- plans ------------------------------------------------------------------
+ * A plan is the new OEG: groups in execution order.  Group g
+ * consists of members[group_begin[g] .. group_begin[g+1]) (statement refs;
+ * listing every statement of a kernel fuses the whole kernel, listing a subset
+ * is fission).  Checks: partition (every statement exactly once), order
+ * (every dependency edge goes forward or stays inside a group), in-group
+ * hazards (reading R11), resources (shared memory, deep-halo depth).  On error
+ * the previous plan stays in place.  Host-side only: generates the kernels'
+ * source; compilation happens in sp_compile or at the first run. */
+sp_status fusion_plan_set(stencil_program *prog, int32_t n_groups, const int32_t *group_begin,
+                          const sp_stmt_ref *members);
+
+/* mode 0 = unfused (one launch per original kernel), 1 = fused plan. */
+sp_status sp_plan_count(const stencil_program *prog, int32_t mode, int32_t *n_launches);
+sp_status sp_plan_report(const stencil_program *prog, int32_t mode, int32_t launch,
+                         sp_group_report *out);
+sp_status fusion_plan_report(const stencil_program *prog, int32_t group, sp_group_report *out);
+/* Generated CUDA source of a mode (for inspection); *len receives the full size. */
+sp_status sp_plan_source(stencil_program *prog, int32_t mode, char *buf, size_t cap, size_t *len);
+/* JIT-compile (NVRTC, sm_100a) without launching; needs no GPU. */
+sp_status sp_compile(stencil_program *prog, int32_t mode);
+
+/* ---- execution ---------------------------------------------------------- */
+/* Every original kernel once, in program order: one launch per kernel, each
+ * reading its inputs from and writing all its outputs to HBM. */
+sp_status run_unfused(stencil_program *prog, sp_stream stream);
+/* The current plan's groups in order (SP_E_STATE if no plan).  On several
+ * ranks each group is preceded by the halo exchange its z-reach needs,
+ * overlapped with the group's interior chunks. */
+sp_status run_fused(stencil_program *prog, sp_stream stream);
+/* One launch of a mode (profiling / per-kernel timing); no exchange. */
+sp_status sp_run_launch(stencil_program *prog, int32_t mode, int32_t launch, sp_stream stream);
+
+/* Exchange `depth` ghost planes of each listed array with the z-neighbours
+ * (ncclSend/ncclRecv grouped; planes are contiguous, no packing).  Requires
+ * a communicator; 1 <= depth <= zhalo. */
+sp_status exchange_halos(stencil_program *prog, int32_t n, const int32_t *arrays, int32_t depth,
+                         sp_stream stream);
+
+const char *sp_last_error(void);
+
+#ifdef __cplusplus
+}
+#endif
+#endif /* STENCILFUSE_H */

@@ -1,0 +1,265 @@
+"""B200-native executor of stencil kernel DAGs with fission/fusion plans.
+
+Thin ctypes binding of libstencilfuse.so (include/stencilfuse.h).  Argument
+marshalling only: every step of the hot path (the generated sm_100a kernels,
+the NCCL halo exchange) runs inside the library.  torch provides device
+memory, streams and the process group; it computes nothing here.  If the
+library is missing, import fails loudly — there is no fallback.
+
+Method: Wahib & Maruyama, "Automated GPU Kernel Transformations in Large-Scale
+Production Stencil Applications", HPDC'15.
+"""
+from __future__ import annotations
+
+import ctypes
+import os
+
+from ._abi import (SP_F32, SP_F64, ROLE, SpArrayDesc, SpEdge, SpGrid, SpGroupReport, SpKernel,
+                   SpLayout, SpStmt, SpStmtRef, SpTerm, SpTap, lib)
+
+__all__ = ["Program", "Comm", "StencilError", "lib"]
+
+
+class StencilError(RuntimeError):
+    def __init__(self, code, msg):
+        super().__init__(f"[sp_status {code}] {msg}")
+        self.code = code
+
+
+def _check(rc):
+    if rc != 0:
+        raise StencilError(rc, lib().sp_last_error().decode())
+
+
+def _stream_handle(stream):
+    if stream is None:
+        import torch
+        stream = torch.cuda.current_stream()
+    if hasattr(stream, "cuda_stream"):
+        return ctypes.c_void_p(stream.cuda_stream)
+    return ctypes.c_void_p(int(stream))
+
+
+class Comm:
+    """NCCL communicator for the z-slab decomposition, bootstrapped over torch.distributed."""
+
+    def __init__(self, rank: int, world: int, group=None):
+        import torch
+        import torch.distributed as dist
+        buf = (ctypes.c_ubyte * 128)()
+        if rank == 0:
+            _check(lib().sp_comm_unique_id(buf))
+        t = torch.tensor(list(bytes(buf)), dtype=torch.uint8)
+        if dist.is_initialized() and world > 1:
+            backend = dist.get_backend(group)
+            dev = torch.device("cuda", torch.cuda.current_device()) if backend == "nccl" else "cpu"
+            t = t.to(dev)
+            dist.broadcast(t, src=0, group=group)
+            t = t.cpu()
+        raw = (ctypes.c_ubyte * 128)(*t.tolist())
+        self.handle = ctypes.c_void_p()
+        _check(lib().sp_comm_create(raw, world, rank, ctypes.byref(self.handle)))
+        self.rank, self.world = rank, world
+
+    def __del__(self):
+        h = getattr(self, "handle", None)
+        if h:
+            lib().sp_comm_destroy(h)
+            self.handle = None
+
+
+def _parse_member(prog, ref):
+    """'K' -> all statements of kernel K; 'K:i' -> statement i of K."""
+    kidx = {k["name"]: i for i, k in enumerate(prog["kernels"])}
+    if ":" in ref:
+        k, s = ref.rsplit(":", 1)
+        return [(kidx[k], int(s))]
+    k = kidx[ref]
+    return [(k, s) for s in range(len(prog["kernels"][k]["stmts"]))]
+
+
+class Program:
+    """A stencil program (kernels over shared 3-D arrays) bound to device memory.
+
+    prog: dict in the synth/programs.py schema.  For a z-slab of a decomposed
+    grid pass nz_global / z_offset / zhalo and a Comm.
+    """
+
+    def __init__(self, prog: dict, comm: Comm | None = None, nz_global=None, z_offset=0,
+                 zhalo=0, options: dict | None = None):
+        self.prog = prog
+        self.dtype = prog["dtype"]
+        g = prog["grid"]
+        self.n = (int(g["nx"]), int(g["ny"]), int(g["nz"]))
+        self.ghost = tuple(int(v) for v in g["ghost"])
+        self.names = [a["name"] for a in prog["arrays"]]
+        self.index = {a: i for i, a in enumerate(self.names)}
+        grid = SpGrid(nx=self.n[0], ny=self.n[1], nz_local=self.n[2],
+                      nz_global=int(nz_global or self.n[2]), z_offset=int(z_offset),
+                      ghost=(ctypes.c_int32 * 3)(*self.ghost), zhalo=int(zhalo),
+                      dtype=SP_F64 if self.dtype == "f64" else SP_F32)
+        arrays = (SpArrayDesc * len(self.names))()
+        self._keep = []
+        for i, a in enumerate(prog["arrays"]):
+            nm = a["name"].encode()
+            self._keep.append(nm)
+            arrays[i].name = nm
+            arrays[i].role = ROLE[a["role"]]
+        kernels = (SpKernel * len(prog["kernels"]))()
+        for ki, k in enumerate(prog["kernels"]):
+            stmts = (SpStmt * len(k["stmts"]))()
+            for si, s in enumerate(k["stmts"]):
+                terms = (SpTerm * len(s["terms"]))()
+                for ti, t in enumerate(s["terms"]):
+                    terms[ti].coef = float(t["c"])
+                    terms[ti].a = self._tap(t["a"])
+                    if "b" in t:
+                        terms[ti].has_b = 1
+                        terms[ti].b = self._tap(t["b"])
+                stmts[si].out = self.index[s["out"]]
+                stmts[si].n_terms = len(s["terms"])
+                stmts[si].terms = terms
+                self._keep.append(terms)
+            nm = k["name"].encode()
+            self._keep += [stmts, nm]
+            kernels[ki].name = nm
+            kernels[ki].n_stmts = len(k["stmts"])
+            kernels[ki].stmts = stmts
+        self.comm = comm
+        self.handle = ctypes.c_void_p()
+        _check(lib().stencil_program_create(ctypes.byref(grid), len(self.names), arrays,
+                                            len(prog["kernels"]), kernels,
+                                            comm.handle if comm else None,
+                                            ctypes.byref(self.handle)))
+        lay = SpLayout()
+        _check(lib().stencil_program_layout(self.handle, ctypes.byref(lay)))
+        self.layout = {f: getattr(lay, f) for f, _ in SpLayout._fields_}
+        self.tensors = {}
+        for k, v in (options or {}).items():
+            self.set_option(k, v)
+
+    def _tap(self, t):
+        return SpTap(self.index[t[0]], int(t[1]), int(t[2]), int(t[3]))
+
+    def __del__(self):
+        h = getattr(self, "handle", None)
+        if h:
+            lib().stencil_program_destroy(h)
+            self.handle = None
+
+    # ---------------------------------------------------------- memory
+    @property
+    def elem(self):
+        return 8 if self.dtype == "f64" else 4
+
+    def alloc_shape(self):
+        L = self.layout
+        return (L["z_alloc"], L["y_alloc"], L["x_pitch"])
+
+    def allocate(self, device, names=None, fill=float("nan")):
+        """Allocate (torch) and bind every array; returns {name: tensor [z][y][x_pitch]}."""
+        import torch
+        dt = torch.float64 if self.dtype == "f64" else torch.float32
+        for name in names or self.names:
+            t = torch.full(self.alloc_shape(), fill, dtype=dt, device=device)
+            self.bind(name, t)
+        return self.tensors
+
+    def bind(self, name, tensor):
+        assert tensor.is_contiguous() and tensor.numel() * tensor.element_size() >= self.layout["bytes"]
+        self.tensors[name] = tensor
+        _check(lib().stencil_program_bind(self.handle, self.index[name],
+                                          ctypes.c_void_p(tensor.data_ptr())))
+
+    def padded_view(self, tensor, hz=None):
+        """View of the dense padded region [nz+2hz][ny+2hy][nx+2hx] (ghost width per side)."""
+        L = self.layout
+        hx, hy, gz = self.ghost
+        hz = gz if hz is None else hz
+        nx, ny, nz = self.n
+        return tensor[L["origin_z"] - hz:L["origin_z"] + nz + hz,
+                      L["origin_y"] - hy:L["origin_y"] + ny + hy,
+                      L["origin_x"] - hx:L["origin_x"] + nx + hx]
+
+    def interior_view(self, tensor):
+        L = self.layout
+        nx, ny, nz = self.n
+        return tensor[L["origin_z"]:L["origin_z"] + nz, L["origin_y"]:L["origin_y"] + ny,
+                      L["origin_x"]:L["origin_x"] + nx]
+
+    # ---------------------------------------------------------- program info
+    def set_option(self, key, value):
+        _check(lib().sp_program_set_option(self.handle, key.encode(), int(value)))
+
+    def edges(self):
+        n = ctypes.c_int32()
+        _check(lib().sp_program_edges(self.handle, 0, None, ctypes.byref(n)))
+        buf = (SpEdge * max(n.value, 1))()
+        _check(lib().sp_program_edges(self.handle, n.value, buf, ctypes.byref(n)))
+        return [(e.frm, e.to, e.kind, e.array) for e in buf[:n.value]]
+
+    def fission(self, kernel):
+        ki = kernel if isinstance(kernel, int) else [k["name"] for k in self.prog["kernels"]].index(kernel)
+        ns = len(self.prog["kernels"][ki]["stmts"])
+        comp = (ctypes.c_int32 * ns)()
+        nc = ctypes.c_int32()
+        _check(lib().sp_fission_components(self.handle, ki, comp, ctypes.byref(nc)))
+        return list(comp), nc.value
+
+    # ---------------------------------------------------------- plans
+    def set_plan(self, groups):
+        """groups: list of lists of member refs ('K' or 'K:i'), in execution order."""
+        begin, members = [0], []
+        for g in groups:
+            for ref in g:
+                members += _parse_member(self.prog, ref)
+            begin.append(len(members))
+        b = (ctypes.c_int32 * len(begin))(*begin)
+        m = (SpStmtRef * len(members))(*[SpStmtRef(k, s) for k, s in members])
+        _check(lib().fusion_plan_set(self.handle, len(groups), b, m))
+
+    def n_launches(self, mode):
+        n = ctypes.c_int32()
+        _check(lib().sp_plan_count(self.handle, self._mode(mode), ctypes.byref(n)))
+        return n.value
+
+    def report(self, mode, i):
+        r = SpGroupReport()
+        _check(lib().sp_plan_report(self.handle, self._mode(mode), i, ctypes.byref(r)))
+        d = {f: getattr(r, f) for f, _ in SpGroupReport._fields_}
+        d["ext"] = list(r.ext)
+        return d
+
+    def reports(self, mode):
+        return [self.report(mode, i) for i in range(self.n_launches(mode))]
+
+    def source(self, mode):
+        n = ctypes.c_size_t()
+        _check(lib().sp_plan_source(self.handle, self._mode(mode), None, 0, ctypes.byref(n)))
+        buf = ctypes.create_string_buffer(n.value + 1)
+        _check(lib().sp_plan_source(self.handle, self._mode(mode), buf, n.value + 1, ctypes.byref(n)))
+        return buf.value.decode()
+
+    def compile(self, mode):
+        _check(lib().sp_compile(self.handle, self._mode(mode)))
+
+    @staticmethod
+    def _mode(mode):
+        return {"unfused": 0, "fused": 1, 0: 0, 1: 1}[mode]
+
+    # ---------------------------------------------------------- execution
+    def run_unfused(self, stream=None):
+        _check(lib().run_unfused(self.handle, _stream_handle(stream)))
+
+    def run_fused(self, stream=None):
+        _check(lib().run_fused(self.handle, _stream_handle(stream)))
+
+    def run(self, mode, stream=None):
+        (self.run_fused if self._mode(mode) else self.run_unfused)(stream)
+
+    def run_launch(self, mode, i, stream=None):
+        _check(lib().sp_run_launch(self.handle, self._mode(mode), i, _stream_handle(stream)))
+
+    def exchange_halos(self, names, depth, stream=None):
+        arr = (ctypes.c_int32 * len(names))(*[self.index[n] for n in names])
+        _check(lib().exchange_halos(self.handle, len(names), arr, depth, _stream_handle(stream)))

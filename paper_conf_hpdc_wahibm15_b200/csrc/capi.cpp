@@ -1,0 +1,330 @@
+// capi.cpp — extern "C" boundary (include/stencilfuse.h) and the executor.
+//
+// Host code of the transformed program (§5.5.4): the new kernels are
+// invoked in the order of the new OEG (plan order).  On several ranks each
+// group is preceded by the z-slab halo exchange of the inputs its z-reach
+// touches; the group's interior chunks do not depend on the exchange and are
+// launched first, so compute overlaps communication.
+#include <cuda_runtime.h>
+
+#include <algorithm>
+#include <cstring>
+
+#include "sf_internal.h"
+
+stencil_program *sf_program_create_impl(const sp_grid *, int32_t, const sp_array_desc *, int32_t,
+                                        const sp_kernel *, sp_comm *);
+void sf_plan_set_impl(stencil_program *, int32_t, const int32_t *, const sp_stmt_ref *);
+void sf_unfused_prepare(stencil_program *);
+sp_comm *sf_comm_create_impl(const void *, int32_t, int32_t);
+void sf_comm_destroy_impl(sp_comm *);
+void sf_comm_unique_id_impl(void *);
+
+namespace sf {
+static thread_local std::string t_err;
+void set_error(const std::string &m) { t_err = m; }
+void fail(sp_status code, const std::string &msg) { throw Error{code, msg}; }
+}  // namespace sf
+
+using namespace sf;
+
+template <class F>
+static sp_status guard(F &&f) {
+    try {
+        f();
+        t_err.clear();
+        return SP_OK;
+    } catch (const Error &e) {
+        t_err = e.msg;
+        return e.code;
+    } catch (const std::bad_alloc &) {
+        t_err = "out of host memory";
+        return SP_E_RESOURCES;
+    } catch (const std::exception &e) {
+        t_err = e.what();
+        return SP_E_ARG;
+    } catch (...) {
+        t_err = "unknown error";
+        return SP_E_ARG;
+    }
+}
+
+static Mode &mode_of(stencil_program *p, int mode) {
+    if (mode == 0) {
+        sf_unfused_prepare(p);
+        return p->unfused;
+    }
+    if (mode == 1) {
+        if (!p->has_plan) fail(SP_E_STATE, "no fusion plan set");
+        return p->fused;
+    }
+    fail(SP_E_ARG, "mode must be 0 (unfused) or 1 (fused)");
+}
+
+// chunks of launch L whose reads stay inside the local slab (no ghost planes
+// exchanged by this group needed): [lo, hi)
+static void interior_chunks(const stencil_program *p, const Launch &L, int *lo, int *hi) {
+    const int64_t nz = p->grid.nz_local;
+    int qlo = 0, ahi = 0;
+    for (const Input &I : L.in) { qlo = std::min(qlo, I.qlo); ahi = std::max(ahi, I.ahi); }
+    int a = L.nch, b = 0;
+    for (int c = 0; c < L.nch; ++c) {
+        int64_t z0 = (int64_t)c * L.zc, z1 = std::min<int64_t>(z0 + L.zc, nz);
+        if (z0 + qlo >= 0 && z1 - 1 + ahi <= nz - 1) { a = std::min(a, c); b = std::max(b, c + 1); }
+    }
+    if (a >= b) { a = 0; b = 0; }
+    *lo = a;
+    *hi = b;
+}
+
+static void run_mode(stencil_program *p, int mode, void *stream) {
+    Mode &m = mode_of(p, mode);
+    load_mode(p, m);
+    const bool multi = p->comm && p->comm->nranks > 1;
+    for (size_t i = 0; i < m.launches.size(); ++i) {
+        Launch &L = m.launches[i];
+        if (L.dead) continue;
+        int depth = std::max(L.z_below, L.z_above);
+        std::vector<int> xarr;
+        for (const Input &I : L.in)
+            if (I.qlo < 0 || I.ahi > 0) xarr.push_back(I.arr);
+        if (!multi || depth == 0 || xarr.empty()) {
+            launch(p, m, (int)i, stream, 0, 1, L.nch);
+            continue;
+        }
+        int lo, hi;
+        interior_chunks(p, L, &lo, &hi);
+        // exchange on the communicator's stream, ordered after prior work on `stream`
+        cudaStream_t cs = (cudaStream_t)p->comm->comm_stream;
+        if (p->events.size() < 2) {
+            for (int e = 0; e < 2; ++e) {
+                cudaEvent_t ev;
+                if (cudaEventCreateWithFlags(&ev, cudaEventDisableTiming) != cudaSuccess)
+                    fail(SP_E_CUDA, "cudaEventCreate");
+                p->events.push_back(ev);
+            }
+        }
+        cudaEvent_t ready = (cudaEvent_t)p->events[0], done = (cudaEvent_t)p->events[1];
+        if (cudaEventRecord(ready, (cudaStream_t)stream) != cudaSuccess ||
+            cudaStreamWaitEvent(cs, ready, 0) != cudaSuccess)
+            fail(SP_E_CUDA, "event record/wait");
+        exchange(p, xarr, depth, cs);
+        if (cudaEventRecord(done, cs) != cudaSuccess) fail(SP_E_CUDA, "event record");
+        if (hi > lo) launch(p, m, (int)i, stream, lo, 1, hi - lo);   // interior: overlaps
+        if (cudaStreamWaitEvent((cudaStream_t)stream, done, 0) != cudaSuccess)
+            fail(SP_E_CUDA, "stream wait");
+        if (lo > 0) launch(p, m, (int)i, stream, 0, 1, lo);
+        if (hi < L.nch) launch(p, m, (int)i, stream, hi, 1, L.nch - hi);
+    }
+}
+
+extern "C" {
+
+const char *sp_last_error(void) { return t_err.c_str(); }
+
+sp_status sp_comm_unique_id(void *out128) {
+    return guard([&] {
+        if (!out128) fail(SP_E_ARG, "null output");
+        sf_comm_unique_id_impl(out128);
+    });
+}
+
+sp_status sp_comm_create(const void *id, int32_t nranks, int32_t rank, sp_comm **out) {
+    return guard([&] {
+        if (!id || !out || nranks < 1 || rank < 0 || rank >= nranks) fail(SP_E_ARG, "bad comm args");
+        *out = sf_comm_create_impl(id, nranks, rank);
+    });
+}
+
+void sp_comm_destroy(sp_comm *c) {
+    if (c) guard([&] { sf_comm_destroy_impl(c); });
+}
+
+sp_status stencil_program_create(const sp_grid *grid, int32_t n_arrays, const sp_array_desc *arrays,
+                                 int32_t n_kernels, const sp_kernel *kernels, sp_comm *comm,
+                                 stencil_program **out) {
+    return guard([&] {
+        if (!out) fail(SP_E_ARG, "null output pointer");
+        *out = nullptr;
+        *out = sf_program_create_impl(grid, n_arrays, arrays, n_kernels, kernels, comm);
+    });
+}
+
+void stencil_program_destroy(stencil_program *p) {
+    if (!p) return;
+    guard([&] {
+        unload_mode(p->unfused);
+        unload_mode(p->fused);
+        for (void *e : p->events) cudaEventDestroy((cudaEvent_t)e);
+    });
+    delete p;
+}
+
+sp_status stencil_program_layout(const stencil_program *p, sp_layout *out) {
+    return guard([&] {
+        if (!p || !out) fail(SP_E_ARG, "null argument");
+        *out = p->layout;
+    });
+}
+
+sp_status stencil_program_bind(stencil_program *p, int32_t array, void *dev_ptr) {
+    return guard([&] {
+        if (!p || array < 0 || array >= (int)p->arrays.size()) fail(SP_E_ARG, "bad array index");
+        if (!dev_ptr || ((uintptr_t)dev_ptr & 255))
+            fail(SP_E_ARG, "device pointer must be non-null and 256-byte aligned");
+        if (p->ptrs[array] != dev_ptr) {
+            p->ptrs[array] = dev_ptr;
+            p->bind_version++;
+        }
+    });
+}
+
+sp_status sp_program_set_option(stencil_program *p, const char *key, int64_t v) {
+    return guard([&] {
+        if (!p || !key) fail(SP_E_ARG, "null argument");
+        std::string k = key;
+        Options &o = p->opt;
+        if (k == "fmad") o.fmad = v != 0;
+        else if (k == "tile_x") o.tile_x = (int)v;
+        else if (k == "tile_y") o.tile_y = (int)v;
+        else if (k == "zchunk") o.zchunk = (int)v;
+        else if (k == "threads") o.threads = (int)v;
+        else if (k == "prefetch") o.prefetch = (int)v;
+        else if (k == "num_sms") p->num_sms = (int)v;
+        else if (k == "loader") o.loader = (int)v;
+        else if (k == "l2_flush") {}
+        else fail(SP_E_ARG, "unknown option '" + k + "'");
+        if (v < 0 && k != "prefetch") fail(SP_E_ARG, "negative option value");
+        if ((k == "threads" && v && (v % 32 || v > 1024)) || (k == "tile_x" && v > 256) ||
+            (k == "tile_y" && v > 256))
+            fail(SP_E_ARG, "option value out of range");
+        // options change code: drop analysed/compiled state (plans are re-analysed)
+        unload_mode(p->unfused);
+        p->unfused = Mode();
+        if (p->has_plan) {
+            Mode m;
+            analyze_mode(p, true, p->plan_groups, m);
+            unload_mode(p->fused);
+            p->fused = std::move(m);
+        }
+    });
+}
+
+sp_status sp_program_counts(const stencil_program *p, int32_t *n_stmts, int32_t *n_edges) {
+    return guard([&] {
+        if (!p) fail(SP_E_ARG, "null program");
+        if (n_stmts) *n_stmts = (int)p->stmts.size();
+        if (n_edges) *n_edges = (int)p->edges.size();
+    });
+}
+
+sp_status sp_program_edges(const stencil_program *p, int32_t cap, sp_edge *out, int32_t *n) {
+    return guard([&] {
+        if (!p || (cap > 0 && !out)) fail(SP_E_ARG, "null argument");
+        int m = std::min<int>(cap, (int)p->edges.size());
+        for (int i = 0; i < m; ++i) out[i] = p->edges[i];
+        if (n) *n = (int)p->edges.size();
+    });
+}
+
+sp_status sp_fission_components(const stencil_program *p, int32_t kernel, int32_t *comp,
+                                int32_t *n_comp) {
+    return guard([&] {
+        if (!p || !comp || !n_comp || kernel < 0 || kernel >= (int)p->kernels.size())
+            fail(SP_E_ARG, "bad argument");
+        int nc = 0;
+        std::vector<int> c = fission_components(p, kernel, &nc);
+        for (size_t i = 0; i < c.size(); ++i) comp[i] = c[i];
+        *n_comp = nc;
+    });
+}
+
+sp_status fusion_plan_set(stencil_program *p, int32_t n_groups, const int32_t *group_begin,
+                          const sp_stmt_ref *members) {
+    return guard([&] {
+        if (!p) fail(SP_E_ARG, "null program");
+        sf_plan_set_impl(p, n_groups, group_begin, members);
+    });
+}
+
+sp_status sp_plan_count(const stencil_program *p, int32_t mode, int32_t *n) {
+    return guard([&] {
+        if (!p || !n) fail(SP_E_ARG, "null argument");
+        *n = (int)mode_of(const_cast<stencil_program *>(p), mode).launches.size();
+    });
+}
+
+sp_status sp_plan_report(const stencil_program *p, int32_t mode, int32_t i, sp_group_report *out) {
+    return guard([&] {
+        if (!p || !out) fail(SP_E_ARG, "null argument");
+        Mode &m = mode_of(const_cast<stencil_program *>(p), mode);
+        if (i < 0 || i >= (int)m.launches.size()) fail(SP_E_ARG, "launch index out of range");
+        fill_report(p, m.launches[i], out);
+    });
+}
+
+sp_status fusion_plan_report(const stencil_program *p, int32_t group, sp_group_report *out) {
+    return sp_plan_report(p, 1, group, out);
+}
+
+sp_status sp_plan_source(stencil_program *p, int32_t mode, char *buf, size_t cap, size_t *len) {
+    return guard([&] {
+        if (!p) fail(SP_E_ARG, "null program");
+        Mode &m = mode_of(p, mode);
+        std::string all;
+        for (const Launch &L : m.launches) all += L.dead ? "// (dead launch " + L.name + ")\n" : L.source;
+        if (len) *len = all.size();
+        if (buf && cap) {
+            size_t n = std::min(cap - 1, all.size());
+            std::memcpy(buf, all.data(), n);
+            buf[n] = 0;
+        }
+    });
+}
+
+sp_status sp_compile(stencil_program *p, int32_t mode) {
+    return guard([&] {
+        if (!p) fail(SP_E_ARG, "null program");
+        compile_mode(p, mode_of(p, mode));
+    });
+}
+
+sp_status run_unfused(stencil_program *p, sp_stream stream) {
+    return guard([&] {
+        if (!p) fail(SP_E_ARG, "null program");
+        run_mode(p, 0, stream);
+    });
+}
+
+sp_status run_fused(stencil_program *p, sp_stream stream) {
+    return guard([&] {
+        if (!p) fail(SP_E_ARG, "null program");
+        run_mode(p, 1, stream);
+    });
+}
+
+sp_status sp_run_launch(stencil_program *p, int32_t mode, int32_t i, sp_stream stream) {
+    return guard([&] {
+        if (!p) fail(SP_E_ARG, "null program");
+        Mode &m = mode_of(p, mode);
+        if (i < 0 || i >= (int)m.launches.size()) fail(SP_E_ARG, "launch index out of range");
+        load_mode(p, m);
+        launch(p, m, i, stream, 0, 1, m.launches[i].nch);
+    });
+}
+
+sp_status exchange_halos(stencil_program *p, int32_t n, const int32_t *arrays, int32_t depth,
+                         sp_stream stream) {
+    return guard([&] {
+        if (!p || n < 0 || (n > 0 && !arrays)) fail(SP_E_ARG, "bad argument");
+        if (!p->comm) fail(SP_E_STATE, "exchange_halos needs a communicator");
+        if (depth < 1 || depth > p->grid.zhalo || depth > p->grid.nz_local)
+            fail(SP_E_ARG, "depth must be in [1, min(zhalo, nz_local)]");
+        std::vector<int> a(arrays, arrays + n);
+        for (int x : a)
+            if (x < 0 || x >= (int)p->arrays.size()) fail(SP_E_ARG, "bad array index");
+        exchange(p, a, depth, stream);
+    });
+}
+
+}  // extern "C"

@@ -1,0 +1,83 @@
+// sf_device.cuh — hand-written sm_100a device primitives of the z-march kernels.
+//
+// Every generated group kernel (codegen.cpp) includes this header: the group
+// body (statement expressions, regions, ring depths) is emitted per plan, the
+// machinery below is fixed.  Inline PTX only; no CUDA headers are needed, so
+// NVRTC compiles it stand-alone for -arch=sm_100a.
+//
+//   * TMA (cp.async.bulk.tensor.3d) stages one x-y plane of an input array over
+//     the tile plus its halo into a shared-memory ring slot; an mbarrier with
+//     expect_tx counts the bytes (SASS: UTMALDG / SYNCS.ARRIVE.TRANS64).
+//   * Consumers wait on the slot's mbarrier phase parity (try_wait loop).
+//   * Streaming stores of live-out results bypass L1.
+#pragma once
+
+typedef unsigned long long sf_u64;
+typedef unsigned int sf_u32;
+
+// 128-byte CUtensorMap, passed by value in __grid_constant__ kernel parameters
+struct __align__(64) SfTmap { sf_u64 w[16]; };
+
+__device__ __forceinline__ sf_u32 sf_smem_addr(const void *p) {
+    return (sf_u32)__cvta_generic_to_shared(p);
+}
+
+__device__ __forceinline__ void sf_mbar_init(sf_u64 *bar, sf_u32 count) {
+    asm volatile("mbarrier.init.shared::cta.b64 [%0], %1;" ::"r"(sf_smem_addr(bar)), "r"(count)
+                 : "memory");
+}
+
+// make mbarrier initialisation visible to the async (TMA) proxy
+__device__ __forceinline__ void sf_fence_mbar_init() {
+    asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
+    asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
+}
+
+__device__ __forceinline__ void sf_mbar_expect_tx(sf_u64 *bar, sf_u32 bytes) {
+    asm volatile("mbarrier.arrive.expect_tx.shared::cta.b64 _, [%0], %1;" ::"r"(sf_smem_addr(bar)),
+                 "r"(bytes)
+                 : "memory");
+}
+
+__device__ __forceinline__ void sf_mbar_wait(sf_u64 *bar, sf_u32 parity) {
+    asm volatile(
+        "{\n\t.reg .pred P1;\n"
+        "SF_WAIT_%=:\n\t"
+        "mbarrier.try_wait.parity.shared::cta.b64 P1, [%0], %1;\n\t"
+        "@!P1 bra SF_WAIT_%=;\n}" ::"r"(sf_smem_addr(bar)),
+        "r"(parity)
+        : "memory");
+}
+
+__device__ __forceinline__ void sf_prefetch_tmap(const SfTmap *m) {
+    asm volatile("prefetch.tensormap [%0];" ::"l"(m) : "memory");
+}
+
+// one plane box (x, y, z are element coordinates in the padded allocation;
+// out-of-range elements are zero-filled by the TMA unit and never consumed)
+__device__ __forceinline__ void sf_tma_load_3d(void *dst, const SfTmap *map, sf_u64 *bar, int x,
+                                               int y, int z) {
+    asm volatile(
+        "cp.async.bulk.tensor.3d.shared::cluster.global.tile.mbarrier::complete_tx::bytes"
+        " [%0], [%1, {%3, %4, %5}], [%2];" ::"r"(sf_smem_addr(dst)),
+        "l"(map), "r"(sf_smem_addr(bar)), "r"(x), "r"(y), "r"(z)
+        : "memory");
+}
+
+// live-out stores: written once, never re-read by this launch
+__device__ __forceinline__ void sf_st(double *p, double v) {
+    asm volatile("st.global.L1::no_allocate.f64 [%0], %1;" ::"l"(p), "d"(v) : "memory");
+}
+__device__ __forceinline__ void sf_st(float *p, float v) {
+    asm volatile("st.global.L1::no_allocate.f32 [%0], %1;" ::"l"(p), "f"(v) : "memory");
+}
+__device__ __forceinline__ double sf_ld(const double *p) {
+    double v;
+    asm volatile("ld.global.nc.f64 %0, [%1];" : "=d"(v) : "l"(p));
+    return v;
+}
+__device__ __forceinline__ float sf_ld(const float *p) {
+    float v;
+    asm volatile("ld.global.nc.f32 %0, [%1];" : "=f"(v) : "l"(p));
+    return v;
+}

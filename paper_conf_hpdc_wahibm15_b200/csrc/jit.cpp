@@ -1,0 +1,271 @@
+// jit.cpp — NVRTC compilation for sm_100a, module loading, TMA descriptors, launches.
+//
+// The generated kernels ("code generation", §3.2.5 and P:L278-296
+// §5.5) are compiled at run time: the program description is the input, so
+// there is no CUDA source to rewrite (the paper's ROSE path).  Each
+// launch is its own NVRTC program, compiled in parallel host threads; cubins
+// are cached in-process by source hash.  Driver entry points come through the
+// runtime (cudaGetDriverEntryPoint), so the library loads on hosts without a
+// GPU and fails with SP_E_CUDA only when a device call is made.
+#include <cuda.h>
+#include <cuda_runtime.h>
+#include <nvrtc.h>
+
+#include <atomic>
+#include <cstdio>
+#include <cstdlib>
+#include <cstring>
+#include <functional>
+#include <thread>
+#include <unordered_map>
+
+#include "sf_internal.h"
+
+namespace sf {
+
+static const char *kDeviceHeader =
+#include "sf_device_embed.inc"
+    ;
+
+struct Drv {
+    CUresult (*ModuleLoadData)(CUmodule *, const void *) = nullptr;
+    CUresult (*ModuleUnload)(CUmodule) = nullptr;
+    CUresult (*ModuleGetFunction)(CUfunction *, CUmodule, const char *) = nullptr;
+    CUresult (*FuncSetAttribute)(CUfunction, CUfunction_attribute, int) = nullptr;
+    CUresult (*FuncGetAttribute)(int *, CUfunction_attribute, CUfunction) = nullptr;
+    CUresult (*LaunchKernel)(CUfunction, unsigned, unsigned, unsigned, unsigned, unsigned,
+                             unsigned, unsigned, CUstream, void **, void **) = nullptr;
+    CUresult (*TensorMapEncodeTiled)(CUtensorMap *, CUtensorMapDataType, cuuint32_t, void *,
+                                     const cuuint64_t *, const cuuint64_t *, const cuuint32_t *,
+                                     const cuuint32_t *, CUtensorMapInterleave,
+                                     CUtensorMapSwizzle, CUtensorMapL2promotion,
+                                     CUtensorMapFloatOOBfill) = nullptr;
+    CUresult (*GetErrorString)(CUresult, const char **) = nullptr;
+    bool ok = false;
+};
+static Drv g_drv;
+static std::mutex g_drv_mu;
+
+static void cuda_check(cudaError_t e, const char *what) {
+    if (e != cudaSuccess)
+        fail(SP_E_CUDA, std::string(what) + ": " + cudaGetErrorString(e));
+}
+
+static void drv_check(CUresult r, const char *what) {
+    if (r != CUDA_SUCCESS) {
+        const char *s = "unknown";
+        if (g_drv.GetErrorString) g_drv.GetErrorString(r, &s);
+        fail(SP_E_CUDA, std::string(what) + ": " + s);
+    }
+}
+
+template <class F>
+static void entry(const char *name, F &fp) {
+    void *ptr = nullptr;
+    cudaDriverEntryPointQueryResult q;
+    cudaError_t e = cudaGetDriverEntryPoint(name, &ptr, cudaEnableDefault, &q);
+    if (e != cudaSuccess || q != cudaDriverEntryPointSuccess || !ptr)
+        fail(SP_E_CUDA, std::string("driver entry point ") + name + " unavailable");
+    fp = reinterpret_cast<F>(ptr);
+}
+
+void ensure_cuda() {
+    std::lock_guard<std::mutex> lk(g_drv_mu);
+    int n = 0;
+    cudaError_t e = cudaGetDeviceCount(&n);
+    if (e != cudaSuccess || n == 0)
+        fail(SP_E_CUDA, std::string("no CUDA device available (") + cudaGetErrorString(e) +
+                            "); this library has no CPU fallback");
+    cuda_check(cudaFree(nullptr), "cudaFree(0) (context init)");
+    if (g_drv.ok) return;
+    entry("cuModuleLoadData", g_drv.ModuleLoadData);
+    entry("cuModuleUnload", g_drv.ModuleUnload);
+    entry("cuModuleGetFunction", g_drv.ModuleGetFunction);
+    entry("cuFuncSetAttribute", g_drv.FuncSetAttribute);
+    entry("cuFuncGetAttribute", g_drv.FuncGetAttribute);
+    entry("cuLaunchKernel", g_drv.LaunchKernel);
+    entry("cuTensorMapEncodeTiled", g_drv.TensorMapEncodeTiled);
+    entry("cuGetErrorString", g_drv.GetErrorString);
+    g_drv.ok = true;
+}
+
+// ------------------------------------------------------------------ NVRTC
+static std::mutex g_cache_mu;
+static std::unordered_map<std::string, std::pair<std::string, int>> g_cache;  // key -> (cubin, regs)
+
+static std::string compile_one(const std::string &src, bool fmad, const std::string &name,
+                               int *regs) {
+    std::string key = std::to_string(std::hash<std::string>{}(src)) + (fmad ? "f" : "n") +
+                      std::to_string(src.size());
+    {
+        std::lock_guard<std::mutex> lk(g_cache_mu);
+        auto it = g_cache.find(key);
+        if (it != g_cache.end()) {
+            *regs = it->second.second;
+            return it->second.first;
+        }
+    }
+    nvrtcProgram prog;
+    const char *hdr_src[] = {kDeviceHeader};
+    const char *hdr_name[] = {"sf_device.cuh"};
+    if (nvrtcCreateProgram(&prog, src.c_str(), (name + ".cu").c_str(), 1, hdr_src, hdr_name) !=
+        NVRTC_SUCCESS)
+        fail(SP_E_JIT, "nvrtcCreateProgram failed");
+    std::vector<const char *> opts = {"-arch=sm_100a", "-std=c++17", "-lineinfo",
+                                      fmad ? "--fmad=true" : "--fmad=false", "--ftz=false",
+                                      "--prec-div=true", "--prec-sqrt=true",
+                                      "--ptxas-options=-v", "-DNDEBUG"};
+    nvrtcResult r = nvrtcCompileProgram(prog, (int)opts.size(), opts.data());
+    size_t log_size = 0;
+    nvrtcGetProgramLogSize(prog, &log_size);
+    std::string log(log_size, '\0');
+    if (log_size) nvrtcGetProgramLog(prog, &log[0]);
+    if (r != NVRTC_SUCCESS) {
+        nvrtcDestroyProgram(&prog);
+        fail(SP_E_JIT, "NVRTC failed for " + name + ": " + log.substr(0, 4000));
+    }
+    size_t n = 0;
+    nvrtcGetCUBINSize(prog, &n);
+    std::string cubin(n, '\0');
+    nvrtcGetCUBIN(prog, &cubin[0]);
+    nvrtcDestroyProgram(&prog);
+    int rr = -1;
+    auto pos = log.find("Used ");
+    if (pos != std::string::npos) rr = std::atoi(log.c_str() + pos + 5);
+    if (log.find("bytes spill stores") != std::string::npos) {
+        auto sp = log.find("bytes spill stores");
+        auto b = log.rfind(',', sp);
+        int spill = std::atoi(log.c_str() + (b == std::string::npos ? 0 : b + 1));
+        if (spill > 0) std::fprintf(stderr, "[stencilfuse] warning: %s spills %d bytes\n",
+                                    name.c_str(), spill);
+    }
+    *regs = rr;
+    if (const char *dir = std::getenv("SF_DUMP_DIR")) {  // debugging aid: source, cubin, log
+        std::string base = std::string(dir) + "/" + name;
+        if (FILE *f = std::fopen((base + ".cu").c_str(), "w")) { std::fwrite(src.data(), 1, src.size(), f); std::fclose(f); }
+        if (FILE *f = std::fopen((base + ".cubin").c_str(), "wb")) { std::fwrite(cubin.data(), 1, cubin.size(), f); std::fclose(f); }
+        if (FILE *f = std::fopen((base + ".log").c_str(), "w")) { std::fwrite(log.data(), 1, log.size(), f); std::fclose(f); }
+    }
+    std::lock_guard<std::mutex> lk(g_cache_mu);
+    g_cache[key] = {cubin, rr};
+    return cubin;
+}
+
+void compile_mode(stencil_program *p, Mode &m) {
+    if (m.compiled) return;
+    const int n = (int)m.launches.size();
+    std::vector<std::string> errs(n);
+    std::atomic<int> next{0};
+    auto work = [&]() {
+        for (;;) {
+            int i = next.fetch_add(1);
+            if (i >= n) return;
+            Launch &L = m.launches[i];
+            if (L.dead) continue;
+            try {
+                L.cubin = compile_one(L.source, p->opt.fmad != 0, L.fn, &L.regs);
+            } catch (const Error &e) {
+                errs[i] = e.msg;
+            }
+        }
+    };
+    int nth = (int)std::min<unsigned>(std::max(1u, std::thread::hardware_concurrency()), 16u);
+    nth = std::min(nth, std::max(n, 1));
+    std::vector<std::thread> th;
+    for (int t = 0; t < nth; ++t) th.emplace_back(work);
+    for (auto &t : th) t.join();
+    for (int i = 0; i < n; ++i)
+        if (!errs[i].empty()) fail(SP_E_JIT, errs[i]);
+    m.compiled = true;
+}
+
+void unload_mode(Mode &m) {
+    if (m.loaded && g_drv.ok)
+        for (Launch &L : m.launches)
+            if (L.module) g_drv.ModuleUnload((CUmodule)L.module);
+    for (Launch &L : m.launches) { L.module = nullptr; L.func = nullptr; }
+    m.loaded = false;
+}
+
+void load_mode(stencil_program *p, Mode &m) {
+    ensure_cuda();
+    if (!m.compiled) compile_mode(p, m);
+    if (m.loaded) return;
+    int dev = 0;
+    cuda_check(cudaGetDevice(&dev), "cudaGetDevice");
+    int sms = 0;
+    cuda_check(cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev), "attr");
+    for (size_t i = 0; i < m.launches.size(); ++i) {
+        Launch &L = m.launches[i];
+        if (L.dead) continue;
+        CUmodule mod;
+        drv_check(g_drv.ModuleLoadData(&mod, L.cubin.data()), "cuModuleLoadData");
+        CUfunction f;
+        drv_check(g_drv.ModuleGetFunction(&f, mod, L.fn.c_str()), "cuModuleGetFunction");
+        drv_check(g_drv.FuncSetAttribute(f, CU_FUNC_ATTRIBUTE_MAX_DYNAMIC_SHARED_SIZE_BYTES,
+                                         (int)L.smem),
+                  "cuFuncSetAttribute(smem)");
+        int regs = 0;
+        g_drv.FuncGetAttribute(&regs, CU_FUNC_ATTRIBUTE_NUM_REGS, f);
+        L.regs = regs;
+        L.module = mod;
+        L.func = f;
+    }
+    m.params.assign(m.launches.size(), {});
+    m.maps_version = ~0ull;
+    m.loaded = true;
+}
+
+static void build_params(stencil_program *p, Mode &m) {
+    if (m.maps_version == p->bind_version) return;
+    const int e = p->elem;
+    const sp_layout &lay = p->layout;
+    for (size_t i = 0; i < m.launches.size(); ++i) {
+        Launch &L = m.launches[i];
+        if (L.dead) continue;
+        std::vector<Mode::Blk> &blk = m.params[i];
+        blk.assign(L.param_size / 64 + 1, Mode::Blk{});
+        unsigned char *buf = blk[0].b;
+        for (size_t a = 0; a < L.in.size(); ++a) {
+            void *ptr = p->ptrs[L.in[a].arr];
+            if (!ptr) fail(SP_E_STATE, "array '" + p->arrays[L.in[a].arr].name + "' is not bound");
+            CUtensorMap tm;
+            cuuint64_t dims[3] = {(cuuint64_t)lay.x_pitch, (cuuint64_t)lay.y_alloc,
+                                  (cuuint64_t)lay.z_alloc};
+            cuuint64_t strides[2] = {(cuuint64_t)(lay.x_pitch * e),
+                                     (cuuint64_t)(lay.x_pitch * lay.y_alloc * e)};
+            cuuint32_t box[3] = {(cuuint32_t)L.in_rw[a], (cuuint32_t)L.in_rh[a], 1};
+            cuuint32_t es[3] = {1, 1, 1};
+            drv_check(g_drv.TensorMapEncodeTiled(
+                          &tm, e == 8 ? CU_TENSOR_MAP_DATA_TYPE_FLOAT64 : CU_TENSOR_MAP_DATA_TYPE_FLOAT32,
+                          3, ptr, dims, strides, box, es, CU_TENSOR_MAP_INTERLEAVE_NONE,
+                          CU_TENSOR_MAP_SWIZZLE_NONE, CU_TENSOR_MAP_L2_PROMOTION_L2_256B,
+                          CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE),
+                      "cuTensorMapEncodeTiled");
+            std::memcpy(buf + 128 * a, &tm, 128);
+        }
+        for (size_t s = 0; s < L.slot_arr.size(); ++s) {
+            void *ptr = p->ptrs[L.slot_arr[s]];
+            if (!ptr) fail(SP_E_STATE, "array '" + p->arrays[L.slot_arr[s]].name + "' is not bound");
+            std::memcpy(buf + L.ptr_off + 8 * s, &ptr, 8);
+        }
+    }
+    m.maps_version = p->bind_version;
+}
+
+void launch(stencil_program *p, Mode &m, int i, void *stream, int chunk_first, int chunk_step,
+            int nchunks) {
+    Launch &L = m.launches[i];
+    if (L.dead || nchunks <= 0) return;
+    build_params(p, m);
+    unsigned char *base = m.params[i][0].b;
+    int32_t ints[2] = {chunk_first, chunk_step};
+    std::memcpy(base + L.int_off, ints, 8);
+    void *args[] = {base};
+    drv_check(g_drv.LaunchKernel((CUfunction)L.func, (unsigned)L.ntx, (unsigned)L.nty,
+                                 (unsigned)nchunks, (unsigned)L.nt, 1, 1, (unsigned)L.smem,
+                                 (CUstream)stream, args, nullptr),
+              "cuLaunchKernel");
+}
+
+}  // namespace sf

@@ -1,0 +1,549 @@
+// plan.cpp — plan legality, per-launch analysis, tile choice, byte/flop model.
+//
+// A fused group is the paper's complex fusion (§5.5.3: producers are
+// evaluated on extra halo layers before the barrier, consumers on the tile
+// after it) combined with simple fusion's input sharing (§5.5.2: each
+// array "target of locality" staged on chip once).  On B200 the vertical
+// direction is marched ("horizontal mapping to CUDA grid and iterating in the
+// vertical direction"): producers run `lead` planes ahead of their
+// consumers, so the z-direction needs no recompute inside a chunk.
+//
+// Readings used: R1 ghost points are loaded, never computed;
+// R5 halo depth = accumulated reach per statement; R6 live-out; R7 staging;
+// R11 in-group hazards; R12 several writers (SSA inside a group).
+#include <algorithm>
+#include <climits>
+#include <cmath>
+#include <cstring>
+#include <set>
+
+#include "sf_internal.h"
+
+namespace sf {
+
+static int64_t rup(int64_t v, int64_t m) { return (v + m - 1) / m * m; }
+
+// ----------------------------------------------------------------- analysis
+static Launch analyze_group(const stencil_program *p, const std::vector<int> &members,
+                            const std::set<int> &stored_gids) {
+    Launch L;
+    L.members = members;
+    const int n = (int)members.size();
+    L.st.resize(n);
+    std::map<int, int> last_writer;   // array -> position
+    std::map<int, int> input_of;      // array -> input index
+    auto resolve = [&](const Tap &t) {
+        auto it = last_writer.find(t.arr);
+        if (it != last_writer.end()) return Src{true, it->second, t.dx, t.dy, t.dz};
+        auto jt = input_of.find(t.arr);
+        if (jt == input_of.end()) {
+            jt = input_of.emplace(t.arr, (int)L.in.size()).first;
+            Input I;
+            I.arr = t.arr;
+            L.in.push_back(I);
+        }
+        return Src{false, jt->second, t.dx, t.dy, t.dz};
+    };
+    for (int m = 0; m < n; ++m) {
+        const Stmt &S = p->stmts[members[m]];
+        Stage &G = L.st[m];
+        G.gid = S.gid;
+        G.out = S.out;
+        for (const Term &t : S.terms) {
+            TermR r;
+            r.coef = t.coef;
+            r.a = resolve(t.a);
+            r.has_b = t.has_b;
+            r.b = t.has_b ? resolve(t.b) : Src{false, -1, 0, 0, 0};
+            G.terms.push_back(r);
+        }
+        last_writer[S.out] = m;
+        G.stored = stored_gids.count(S.gid) > 0;
+    }
+
+    // backward pass (reading R5): regions, plane ranges, leads
+    const int NEG = INT_MIN / 4;
+    struct Acc { int ex0, ex1, ey0, ey1, loff, lead, minread; bool any; };
+    std::vector<Acc> acc(n, Acc{NEG, NEG, NEG, NEG, INT_MAX / 4, NEG, INT_MAX / 4, false});
+    struct IAcc { int ex0, ex1, ey0, ey1, alo, ahi, qlo; bool any; };
+    std::vector<IAcc> iacc(L.in.size(), IAcc{NEG, NEG, NEG, NEG, INT_MAX / 4, NEG, INT_MAX / 4, false});
+    for (int m = n - 1; m >= 0; --m) {
+        Stage &G = L.st[m];
+        Acc &A = acc[m];
+        if (G.stored) {  // live-out: the tile and the chunk's own planes (R6)
+            A.ex0 = std::max(A.ex0, 0); A.ex1 = std::max(A.ex1, 0);
+            A.ey0 = std::max(A.ey0, 0); A.ey1 = std::max(A.ey1, 0);
+            A.loff = std::min(A.loff, 0); A.lead = std::max(A.lead, 0);
+            A.minread = std::min(A.minread, 0);
+            A.any = true;
+        }
+        if (!A.any) continue;  // dead: nothing consumes it
+        G.needed = true;
+        G.ex0 = A.ex0; G.ex1 = A.ex1; G.ey0 = A.ey0; G.ey1 = A.ey1;
+        G.loff = A.loff; G.lead = A.lead;
+        G.depth = G.lead - std::min(A.minread, G.lead) + 1;
+        for (const TermR &t : G.terms) {
+            for (int w = 0; w < 2; ++w) {
+                if (w == 1 && !t.has_b) continue;
+                const Src &s = w ? t.b : t.a;
+                if (s.stage) {
+                    Acc &P = acc[s.idx];
+                    P.ex0 = std::max(P.ex0, G.ex0 - s.dx); P.ex1 = std::max(P.ex1, G.ex1 + s.dx);
+                    P.ey0 = std::max(P.ey0, G.ey0 - s.dy); P.ey1 = std::max(P.ey1, G.ey1 + s.dy);
+                    P.loff = std::min(P.loff, G.loff + s.dz);
+                    P.lead = std::max(P.lead, G.lead + s.dz);
+                    P.minread = std::min(P.minread, G.lead + s.dz);
+                    P.any = true;
+                } else {
+                    IAcc &I = iacc[s.idx];
+                    I.ex0 = std::max(I.ex0, G.ex0 - s.dx); I.ex1 = std::max(I.ex1, G.ex1 + s.dx);
+                    I.ey0 = std::max(I.ey0, G.ey0 - s.dy); I.ey1 = std::max(I.ey1, G.ey1 + s.dy);
+                    I.alo = std::min(I.alo, G.lead + s.dz);
+                    I.ahi = std::max(I.ahi, G.lead + s.dz);
+                    I.qlo = std::min(I.qlo, G.loff + s.dz);
+                    I.any = true;
+                }
+            }
+        }
+    }
+    // inputs not read by any needed stage are dropped
+    std::vector<int> remap(L.in.size(), -1);
+    std::vector<Input> ins;
+    for (size_t i = 0; i < L.in.size(); ++i) {
+        if (!iacc[i].any) continue;
+        Input I = L.in[i];
+        I.ex0 = iacc[i].ex0; I.ex1 = iacc[i].ex1; I.ey0 = iacc[i].ey0; I.ey1 = iacc[i].ey1;
+        I.alo = iacc[i].alo; I.ahi = iacc[i].ahi; I.qlo = iacc[i].qlo;
+        remap[i] = (int)ins.size();
+        ins.push_back(I);
+    }
+    for (Stage &G : L.st)
+        for (TermR &t : G.terms) {
+            if (!t.a.stage) t.a.idx = remap[t.a.idx];
+            if (t.has_b && !t.b.stage) t.b.idx = remap[t.b.idx];
+        }
+    L.in = ins;
+
+    // storage class (reading R7): register if every consumer reads it at
+    // (0,0,dz) over exactly its own region, else a shared-memory plane ring
+    std::vector<bool> reg_ok(n, true);
+    for (int m = 0; m < n; ++m) {
+        const Stage &G = L.st[m];
+        if (!G.needed) continue;
+        for (const TermR &t : G.terms)
+            for (int w = 0; w < 2; ++w) {
+                if (w == 1 && !t.has_b) continue;
+                const Src &s = w ? t.b : t.a;
+                if (!s.stage) continue;
+                const Stage &P = L.st[s.idx];
+                if (s.dx || s.dy || P.ex0 != G.ex0 || P.ex1 != G.ex1 || P.ey0 != G.ey0 ||
+                    P.ey1 != G.ey1)
+                    reg_ok[s.idx] = false;
+            }
+    }
+    L.kfirst = 0;
+    for (int m = 0; m < n; ++m) {
+        Stage &G = L.st[m];
+        if (!G.needed) { G.keep = Keep::Dead; continue; }
+        G.keep = reg_ok[m] ? Keep::Reg : Keep::Smem;
+        L.kfirst = std::min(L.kfirst, G.loff - G.lead);
+        int c = -1;
+        for (size_t i = 0; i < L.cls.size(); ++i)
+            if (L.cls[i].x0 == -G.ex0 && L.cls[i].x1 == G.ex1 && L.cls[i].y0 == -G.ey0 &&
+                L.cls[i].y1 == G.ey1)
+                c = (int)i;
+        if (c < 0) {
+            c = (int)L.cls.size();
+            L.cls.push_back(RegionClass{-G.ex0, G.ex1, -G.ey0, G.ey1});  // x1/y1 are extensions
+        }
+        G.cls = c;
+    }
+    L.dead = true;
+    for (const Stage &G : L.st) if (G.needed) L.dead = false;
+
+    // z reach for the halo exchange
+    L.z_below = 0;
+    L.z_above = 0;
+    for (const Input &I : L.in) {
+        L.z_below = std::max(L.z_below, -I.qlo);
+        L.z_above = std::max(L.z_above, I.ahi);
+    }
+
+    // R11: a group must not read from HBM an array it stores, except for a
+    // point-wise read of the CTA's own tile and chunk that happens no later
+    // than the store.
+    for (int m = 0; m < n; ++m) {
+        const Stage &W = L.st[m];
+        if (!W.stored) continue;
+        for (int r = 0; r < n; ++r) {
+            const Stage &R = L.st[r];
+            if (!R.needed) continue;
+            for (const TermR &t : R.terms)
+                for (int w = 0; w < 2; ++w) {
+                    if (w == 1 && !t.has_b) continue;
+                    const Src &s = w ? t.b : t.a;
+                    if (s.stage || L.in[s.idx].arr != W.out) continue;
+                    // the reader computes exactly the CTA's own tile x chunk (no halo,
+                    // no warm-up plane, no plane of the next chunk) and reads the
+                    // point it computes; then it reads before any CTA stores there
+                    // iff it runs no later than the store: same step (both leads 0)
+                    bool ok = s.dx == 0 && s.dy == 0 && s.dz == 0 && R.ex0 == 0 && R.ex1 == 0 &&
+                              R.ey0 == 0 && R.ey1 == 0 && R.loff == 0 && R.lead == 0 &&
+                              W.lead == 0;
+                    // same step: R precedes W in program order, but runs on another
+                    // thread when W's region differs from the tile -> barrier first
+                    bool ok2 = W.ex0 == 0 && W.ex1 == 0 && W.ey0 == 0 && W.ey1 == 0;
+                    if (!ok)
+                        fail(SP_E_PLAN_HAZARD,
+                             "statement " + std::to_string(R.gid) + " reads '" +
+                                 p->arrays[W.out].name + "' from memory while statement " +
+                                 std::to_string(W.gid) + " of the same group stores it "
+                                 "(reading R11)");
+                    if (!ok2) L.st[m].war_barrier = true;
+                }
+        }
+    }
+    return L;
+}
+
+// -------------------------------------------------------- config and model
+struct Cost { double t; int64_t smem; };
+
+static void layout_launch(const stencil_program *p, Launch &L) {
+    if (L.tx % (16 / p->elem)) fail(SP_E_ARG, "tile_x must be a multiple of 16 bytes");
+    const int e = p->elem;
+    L.rw_pad = 16 / e;  // TMA: inner box extent multiple of 16 B
+    L.in_off.clear(); L.in_plane.clear(); L.in_rw.clear(); L.in_rh.clear();
+    L.st_off.clear(); L.st_plane.clear(); L.st_w.clear(); L.st_h.clear();
+    int64_t off = 0;
+    L.n_bars = 0;
+    for (Input &I : L.in) {
+        // the innermost start coordinate of a TMA box must be 16-B aligned: the tile
+        // origin is, so round the left extension up to 16 B
+        I.bx0 = (int)rup(std::max(I.ex0, 0), L.rw_pad);
+        int rw = (int)rup(L.tx + I.bx0 + std::max(I.ex1, 0), L.rw_pad);
+        int rh = L.ty + I.ey0 + I.ey1;
+        int64_t plane = rup((int64_t)rw * rh, 128 / e);
+        int D = I.ahi - I.alo + 1 + L.pf;
+        L.in_off.push_back(off);
+        L.in_plane.push_back(plane);
+        L.in_rw.push_back(rw);
+        L.in_rh.push_back(rh);
+        off += plane * D * e;
+        L.n_bars += D;
+    }
+    for (const Stage &G : L.st) {
+        int w = L.tx + G.ex0 + G.ex1, h = L.ty + G.ey0 + G.ey1;
+        L.st_w.push_back(w);
+        L.st_h.push_back(h);
+        if (G.keep == Keep::Smem) {
+            int64_t plane = rup((int64_t)w * h, 128 / e);
+            L.st_off.push_back(off);
+            L.st_plane.push_back(plane);
+            off += plane * G.depth * e;
+        } else {
+            L.st_off.push_back(-1);
+            L.st_plane.push_back(0);
+        }
+    }
+    off = rup(off, 8);
+    L.bar_off = off;
+    off += 8 * (int64_t)L.n_bars;
+    L.smem = rup(off, 128);
+}
+
+// per-point byte/flop model of a configured launch
+static void model(const stencil_program *p, Launch &L) {
+    const int e = p->elem;
+    const double tile = (double)L.tx * L.ty * L.zc;
+    int n_store = 0;
+    double fl_alg = 0, fl_exec = 0, sm = 0;
+    for (const Stage &G : L.st) {
+        if (!G.needed) continue;
+        if (G.stored) ++n_store;
+        int prods = 0;
+        for (const TermR &t : G.terms) prods += t.has_b;
+        double f = 2.0 * G.terms.size() - 1 + prods;
+        fl_alg += f;
+        double pts = (double)(L.tx + G.ex0 + G.ex1) * (L.ty + G.ey0 + G.ey1) *
+                     (L.zc - 1 + G.lead - G.loff + 1);
+        fl_exec += f * pts / tile;
+        int smem_reads = 0;
+        for (const TermR &t : G.terms)
+            for (int w = 0; w < 2; ++w) {
+                if (w == 1 && !t.has_b) continue;
+                const Src &s = w ? t.b : t.a;
+                if (!s.stage || L.st[s.idx].keep == Keep::Smem) ++smem_reads;
+            }
+        sm += (smem_reads + (G.keep == Keep::Smem ? 1 : 0)) * e * pts / tile;
+    }
+    double by_exec = n_store * (double)e;
+    for (size_t i = 0; i < L.in.size(); ++i) {
+        const Input &I = L.in[i];
+        double planes = (L.zc - 1 + I.ahi) - I.qlo + 1;
+        double b = (double)L.in_rw[i] * L.in_rh[i] * planes * e / tile;
+        by_exec += b;
+        sm += b;  // TMA writes into shared memory
+    }
+    L.bytes_alg = (double)e * (L.in.size() + n_store);
+    L.flops_alg = fl_alg;
+    L.flops_exec = fl_exec;
+    L.bytes_exec = by_exec;
+    L.smem_pt = sm;
+}
+
+static int max_region_points(const Launch &L) {
+    int m = 0;
+    for (const Stage &G : L.st)
+        if (G.needed) m = std::max(m, (L.tx + G.ex0 + G.ex1) * (L.ty + G.ey0 + G.ey1));
+    return m;
+}
+
+static void choose_config(const stencil_program *p, Launch &L) {
+    const sp_grid &g = p->grid;
+    const int e = p->elem;
+    const int64_t nz = g.nz_local;
+    std::vector<int> cx, cy, cz, cn, cp;
+    if (p->opt.tile_x) cx = {p->opt.tile_x};
+    else cx = e == 8 ? std::vector<int>{16, 32, 64} : std::vector<int>{32, 64, 128};
+    if (p->opt.tile_y) cy = {p->opt.tile_y};
+    else cy = {1, 2, 4, 8, 16, 32};
+    if (p->opt.zchunk) cz = {p->opt.zchunk};
+    else cz = {4, 8, 16, 32, 64, 128, 256, 512};
+    if (p->opt.threads) cn = {p->opt.threads};
+    else cn = {128, 256, 512};
+    if (p->opt.prefetch >= 0) cp = {p->opt.prefetch};
+    else cp = {1, 2, 3};
+    const double sms = p->num_sms;
+    const double clk = 1.8e9;
+    const double hbm = 6.0e12, smem_bw = sms * 128 * clk;
+    const double alu = sms * (e == 8 ? 64 : 128) * clk;
+    Launch best;
+    double best_t = 1e300;
+    for (int tx : cx) {
+        if (!p->opt.tile_x && tx >= 2 * g.nx && tx != cx.front()) continue;
+        for (int ty : cy) {
+            if (!p->opt.tile_y && ty >= 2 * g.ny && ty != cy.front()) continue;
+            for (int zc : cz) {
+                if (!p->opt.zchunk && zc >= 2 * nz && zc != cz.front()) continue;
+                for (int pf : cp) {
+                    Launch C = L;
+                    C.tx = tx; C.ty = ty; C.zc = (int)std::min<int64_t>(zc, nz); C.pf = pf;
+                    layout_launch(p, C);
+                    if (C.smem > 227 * 1024) continue;
+                    bool box_ok = true;  // TMA box extents are limited to 256
+                    for (size_t i = 0; i < C.in.size(); ++i)
+                        if (C.in_rw[i] > 256 || C.in_rh[i] > 256) box_ok = false;
+                    if (!box_ok) continue;
+                    model(p, C);
+                    int mrp = max_region_points(C);
+                    for (int nt : cn) {
+                        if (!p->opt.threads && nt > rup(mrp, 32) && nt != cn.front()) continue;
+                        C.nt = nt;
+                        C.ntx = (int)((g.nx + tx - 1) / tx);
+                        C.nty = (int)((g.ny + ty - 1) / ty);
+                        C.nch = (int)((nz + C.zc - 1) / C.zc);
+                        double ctas = (double)C.ntx * C.nty * C.nch;
+                        int per_sm = (int)std::min<int64_t>(
+                            {(int64_t)(228 * 1024 / (C.smem + 1024)), (int64_t)(2048 / nt), 32,
+                             (int64_t)(65536 / (nt * 64))});
+                        if (per_sm < 1) continue;
+                        double slots = sms * per_sm;
+                        double waves = std::ceil(ctas / slots);
+                        double fill = ctas / (waves * slots);
+                        double pts = (double)g.nx * g.ny * nz;
+                        double t_mem = C.bytes_exec * pts / hbm;
+                        double t_sm = C.smem_pt * pts / smem_bw;
+                        double t_alu = C.flops_exec * pts / alu;
+                        // idle lanes: points per thread rounding
+                        double lanes = 0, used = 0;
+                        for (const Stage &G : C.st) {
+                            if (!G.needed) continue;
+                            double rp = (double)(tx + G.ex0 + G.ex1) * (ty + G.ey0 + G.ey1);
+                            used += rp;
+                            lanes += std::ceil(rp / nt) * nt;
+                        }
+                        t_alu *= lanes / std::max(used, 1.0);
+                        double t = std::max({t_mem, t_sm, t_alu}) / fill;
+                        // bytes in flight per SM (latency hiding): want >= 32 KB
+                        double inflight = 0;
+                        for (size_t i = 0; i < C.in.size(); ++i)
+                            inflight += (double)C.in_plane[i] * e * pf;
+                        inflight *= std::min<double>(per_sm, std::ceil(ctas / sms));
+                        if (inflight < 32768) t *= 32768.0 / std::max(inflight, 1024.0);
+                        // warps per SM for the compute part
+                        double warps = std::min<double>(per_sm, std::ceil(ctas / sms)) * nt / 32;
+                        if (warps < 8) t *= 8.0 / warps;
+                        t += 2e-6 * waves;  // launch + wave tail overheads
+                        if (t < best_t) { best_t = t; best = C; }
+                    }
+                }
+            }
+        }
+    }
+    if (best_t >= 1e299)
+        fail(SP_E_RESOURCES, "group '" + L.name + "': no tile configuration fits in 227 KB of "
+                             "shared memory (split the group: fission/fusion plan)");
+    L = best;
+}
+
+// ---------------------------------------------------------------- plans
+static void live_out(const stencil_program *p, bool fused,
+                     const std::vector<std::vector<int>> &groups, std::vector<std::set<int>> &stored) {
+    stored.assign(groups.size(), {});
+    const int na = (int)p->arrays.size();
+    if (!fused) {
+        // original kernel: every array it writes goes to memory (last writer)
+        for (size_t g = 0; g < groups.size(); ++g) {
+            std::map<int, int> last;
+            for (int gid : groups[g]) last[p->stmts[gid].out] = gid;
+            for (auto &kv : last) stored[g].insert(kv.second);
+        }
+        return;
+    }
+    // reading R6: X written in G is stored iff a later group reads X from
+    // memory before any rewrite, or X is OUT/INOUT and G holds its last writer.
+    std::vector<std::pair<int, int>> lastw(na, {-1, -1});  // (group, gid)
+    for (size_t g = 0; g < groups.size(); ++g) {
+        std::set<int> written_here;
+        for (int gid : groups[g]) {
+            const Stmt &S = p->stmts[gid];
+            for (const Term &t : S.terms)
+                for (int w = 0; w < 2; ++w) {
+                    if (w == 1 && !t.has_b) continue;
+                    int a = w ? t.b.arr : t.a.arr;
+                    if (written_here.count(a)) continue;  // on-chip value
+                    if (lastw[a].first >= 0 && lastw[a].first < (int)g)
+                        stored[lastw[a].first].insert(lastw[a].second);
+                }
+            written_here.insert(S.out);
+        }
+        std::map<int, int> last;
+        for (int gid : groups[g]) last[p->stmts[gid].out] = gid;
+        for (auto &kv : last) lastw[kv.first] = {(int)g, kv.second};
+    }
+    for (int a = 0; a < na; ++a)
+        if ((p->arrays[a].role == SP_OUT || p->arrays[a].role == SP_INOUT) && lastw[a].first >= 0)
+            stored[lastw[a].first].insert(lastw[a].second);
+}
+
+void analyze_mode(stencil_program *p, bool fused, const std::vector<std::vector<int>> &groups,
+                  Mode &out) {
+    std::vector<std::set<int>> stored;
+    live_out(p, fused, groups, stored);
+    Mode m;
+    for (size_t g = 0; g < groups.size(); ++g) {
+        Launch L = analyze_group(p, groups[g], stored[g]);
+        if (fused) {
+            L.name = "group" + std::to_string(g);
+        } else {
+            L.name = p->kernels[p->stmts[groups[g][0]].kernel].name;
+        }
+        if (p->comm && p->comm->nranks > 1 &&
+            (L.z_below > p->grid.zhalo || L.z_above > p->grid.zhalo))
+            fail(SP_E_RESOURCES, L.name + ": accumulated z-reach " +
+                                     std::to_string(std::max(L.z_below, L.z_above)) +
+                                     " exceeds zhalo " + std::to_string(p->grid.zhalo));
+        if (!L.dead) {
+            choose_config(p, L);
+            model(p, L);
+        }
+        m.launches.push_back(std::move(L));
+    }
+    for (size_t i = 0; i < m.launches.size(); ++i)
+        if (!m.launches[i].dead) generate_launch(p, m.launches[i], (int)i, fused);
+    m.analyzed = true;
+    out = std::move(m);
+}
+
+void fill_report(const stencil_program *p, const Launch &L, sp_group_report *r) {
+    std::memset(r, 0, sizeof(*r));
+    for (const Stage &G : L.st) {
+        if (!G.needed) continue;
+        r->n_stmts++;
+        if (G.stored) r->n_stores++;
+        if (G.keep == Keep::Smem) r->n_smem_stages++;
+        if (G.keep == Keep::Reg) r->n_reg_stages++;
+        r->ext[0] = std::max(r->ext[0], G.ex0);
+        r->ext[1] = std::max(r->ext[1], G.ex1);
+        r->ext[2] = std::max(r->ext[2], G.ey0);
+        r->ext[3] = std::max(r->ext[3], G.ey1);
+    }
+    r->n_inputs = (int)L.in.size();
+    r->z_below = L.z_below;
+    r->z_above = L.z_above;
+    r->tile_x = L.tx;
+    r->tile_y = L.ty;
+    r->zchunk = L.zc;
+    r->threads = L.nt;
+    r->grid_ctas = L.ntx * L.nty * L.nch;
+    r->regs_per_thread = L.regs;
+    r->smem_bytes = L.smem;
+    r->bytes_alg = L.bytes_alg;
+    r->flops_alg = L.flops_alg;
+    r->bytes_exec = L.bytes_exec;
+    r->flops_exec = L.flops_exec;
+    r->smem_bytes_pt = L.smem_pt;
+    (void)p;
+}
+
+}  // namespace sf
+
+// --------------------------------------------------------- plan validation
+using namespace sf;
+
+void sf_plan_set_impl(stencil_program *p, int32_t n_groups, const int32_t *group_begin,
+                      const sp_stmt_ref *members) {
+    if (n_groups <= 0 || !group_begin || !members) fail(SP_E_ARG, "fusion_plan_set: empty plan");
+    const int ns = (int)p->stmts.size();
+    std::vector<int> group_of(ns, -1);
+    std::vector<std::vector<int>> groups(n_groups);
+    if (group_begin[0] != 0) fail(SP_E_ARG, "group_begin[0] must be 0");
+    for (int g = 0; g < n_groups; ++g) {
+        if (group_begin[g + 1] <= group_begin[g]) fail(SP_E_ARG, "empty group in plan");
+        for (int i = group_begin[g]; i < group_begin[g + 1]; ++i) {
+            const sp_stmt_ref &r = members[i];
+            if (r.kernel < 0 || r.kernel >= (int)p->kernels.size())
+                fail(SP_E_ARG, "plan member: kernel index out of range");
+            const Kernel &K = p->kernels[r.kernel];
+            if (r.stmt < 0 || r.stmt >= (int)K.stmts.size())
+                fail(SP_E_ARG, "plan member: statement index out of range");
+            int gid = K.stmts[r.stmt];
+            if (group_of[gid] >= 0)
+                fail(SP_E_PLAN_PARTITION, "statement " + K.name + ":" + std::to_string(r.stmt) +
+                                              " appears twice in the plan");
+            group_of[gid] = g;
+            groups[g].push_back(gid);
+        }
+        std::sort(groups[g].begin(), groups[g].end());  // program order inside a group
+    }
+    for (int s = 0; s < ns; ++s)
+        if (group_of[s] < 0) {
+            const Stmt &S = p->stmts[s];
+            fail(SP_E_PLAN_PARTITION, "statement " + p->kernels[S.kernel].name + ":" +
+                                          std::to_string(S.local) + " is missing from the plan");
+        }
+    // order: every dependency edge must go forward in the new OEG
+    for (const sp_edge &e : p->edges)
+        if (group_of[e.from] > group_of[e.to]) {
+            const Stmt &A = p->stmts[e.from], &B = p->stmts[e.to];
+            fail(SP_E_PLAN_ORDER, "dependency " + p->kernels[A.kernel].name + ":" +
+                                      std::to_string(A.local) + " -> " +
+                                      p->kernels[B.kernel].name + ":" + std::to_string(B.local) +
+                                      " (array '" + p->arrays[e.array].name +
+                                      "') runs backwards in the plan");
+        }
+    Mode m;
+    analyze_mode(p, true, groups, m);  // throws on hazards / resources; old plan kept
+    unload_mode(p->fused);
+    p->fused = std::move(m);
+    p->plan_groups = groups;
+    p->has_plan = true;
+}
+
+void sf_unfused_prepare(stencil_program *p) {
+    if (p->unfused.analyzed) return;
+    std::vector<std::vector<int>> groups;
+    for (const Kernel &K : p->kernels) groups.push_back(K.stmts);
+    analyze_mode(p, false, groups, p->unfused);
+}

@@ -1,0 +1,172 @@
+// sf_internal.h — internal model of the stencil-DAG executor (host side).
+//
+// Program model: kernels, arrays, statements and their dependency edges are the
+// paper's DDG/OEG (§2, §3.2.3).  A Launch is one generated
+// kernel: a fused group of the plan ("new kernel") or one
+// original kernel in unfused mode ("no fusion", §5.5.1).
+#pragma once
+
+#include <cstdint>
+#include <map>
+#include <memory>
+#include <mutex>
+#include <string>
+#include <vector>
+
+#include "stencilfuse.h"
+
+namespace sf {
+
+struct Tap { int arr, dx, dy, dz; };
+struct Term { double coef; Tap a; bool has_b; Tap b; };
+struct Stmt {
+    int kernel, local, gid;  // kernel index, index inside kernel, global program-order id
+    int out;
+    std::vector<Term> terms;
+};
+struct Kernel { std::string name; std::vector<int> stmts; };
+struct ArrayDesc { std::string name; sp_role role; };
+
+struct Options {
+    int fmad = 1;
+    int tile_x = 0, tile_y = 0, zchunk = 0, threads = 0, prefetch = -1;
+    int loader = 0;  // 0: TMA + mbarrier ring, 1: cooperative ld.global -> st.shared
+};
+
+// ---------------------------------------------------------------- analysis
+enum class Keep { Dead, Reg, Smem };
+
+// A term operand after resolution inside a launch: an on-chip stage (position
+// in the launch) or an external input (index into Launch::in).
+struct Src { bool stage; int idx; int dx, dy, dz; };
+struct TermR { double coef; Src a; bool has_b; Src b; };
+
+struct Stage {
+    int gid = -1;           // statement
+    int out = -1;           // array written
+    std::vector<TermR> terms;
+    bool stored = false;    // written back to HBM (live-out, reading R6)
+    bool needed = false;    // computed at all
+    // computed region relative to the tile: x in [-ex0, TX+ex1), y in [-ey0, TY+ey1)
+    int ex0 = 0, ex1 = 0, ey0 = 0, ey1 = 0;
+    // computed planes [loff, zc-1+lead] relative to the chunk; computed at step k: plane k+lead
+    int loff = 0, lead = 0;
+    int depth = 1;          // planes kept on chip (ring / queue)
+    Keep keep = Keep::Dead;
+    int cls = -1;           // region class (thread->point mapping)
+    bool war_barrier = false;  // needs a CTA barrier before its store (R11 exception)
+};
+
+struct Input {
+    int arr = -1;
+    int ex0 = 0, ex1 = 0, ey0 = 0, ey1 = 0;  // region relative to the tile
+    int alo = 0, ahi = 0;   // planes read at step k: [k+alo, k+ahi]
+    int qlo = 0;            // first plane needed (relative to chunk); last = zc-1+ahi
+    int bx0 = 0;            // box x extension, ex0 rounded up to 16 B (TMA box start alignment)
+};
+
+struct RegionClass { int x0, x1, y0, y1; };  // relative to the tile, half-open
+
+struct Launch {
+    std::string name;
+    std::vector<int> members;  // statement gids, program order
+    std::vector<Stage> st;
+    std::vector<Input> in;
+    std::vector<RegionClass> cls;
+    std::vector<int> arr_slot;   // array id -> pointer slot in params (-1 unused)
+    std::vector<int> slot_arr;   // pointer slot -> array id
+    int kfirst = 0;              // first step (<= 0), relative to the chunk
+    int z_below = 0, z_above = 0;
+    // configuration
+    int tx = 0, ty = 0, zc = 0, nt = 0, pf = 0;
+    int ntx = 0, nty = 0, nch = 0;
+    int64_t smem = 0;
+    int rw_pad = 2;              // input row padding granularity (elements)
+    // layout of smem (bytes) per input ring / stage ring
+    std::vector<int64_t> in_off, in_plane;   // plane size in elements (padded)
+    std::vector<int> in_rw, in_rh;
+    std::vector<int64_t> st_off, st_plane;
+    std::vector<int> st_w, st_h;
+    int64_t bar_off = 0;
+    int n_bars = 0;
+    // report
+    double bytes_alg = 0, flops_alg = 0, bytes_exec = 0, flops_exec = 0, smem_pt = 0;
+    // jit
+    std::string fn;
+    std::string source;
+    std::string cubin;
+    int regs = -1;
+    void *func = nullptr;    // CUfunction
+    void *module = nullptr;  // CUmodule
+    size_t param_size = 0, ptr_off = 0, int_off = 0;
+    bool dead = false;       // nothing to compute (all stages dead)
+};
+
+struct Mode {
+    std::vector<Launch> launches;
+    bool analyzed = false;
+    bool compiled = false;
+    bool loaded = false;
+    uint64_t maps_version = ~0ull;
+    struct alignas(64) Blk { unsigned char b[64]; };
+    std::vector<std::vector<Blk>> params;  // per launch: tensor maps + pointers + ints
+};
+
+}  // namespace sf
+
+struct sp_comm_s {
+    void *nccl = nullptr;  // ncclComm_t
+    int nranks = 1, rank = 0, device = 0;
+    void *comm_stream = nullptr;  // cudaStream_t used for exchanges
+};
+
+struct stencil_program_s {
+    sp_grid grid{};
+    int elem = 8;
+    std::vector<sf::ArrayDesc> arrays;
+    std::vector<sf::Kernel> kernels;
+    std::vector<sf::Stmt> stmts;
+    std::vector<sp_edge> edges;
+    sp_layout layout{};
+    int64_t plane = 0;           // x_pitch * y_alloc
+    int64_t zint_lo = 0, zint_hi = 0;  // global interior in local z coordinates
+    std::vector<void *> ptrs;
+    uint64_t bind_version = 0;
+    sp_comm *comm = nullptr;
+    sf::Options opt;
+    sf::Mode unfused, fused;
+    bool has_plan = false;
+    std::vector<std::vector<int>> plan_groups;  // gids per group
+    int num_sms = 148;
+    std::vector<void *> events;  // cudaEvent_t pool for exchange overlap
+};
+
+namespace sf {
+// errors --------------------------------------------------------------------
+void set_error(const std::string &msg);
+struct Error { sp_status code; std::string msg; };
+[[noreturn]] void fail(sp_status code, const std::string &msg);
+
+// program.cpp
+void build_edges(stencil_program *p);
+std::vector<int> fission_components(const stencil_program *p, int kernel, int *n_comp);
+
+// plan.cpp
+void analyze_mode(stencil_program *p, bool fused, const std::vector<std::vector<int>> &groups,
+                  Mode &out);
+void fill_report(const stencil_program *p, const Launch &L, sp_group_report *r);
+
+// codegen.cpp
+std::string generate_launch(const stencil_program *p, Launch &L, int index, bool fused);
+
+// jit.cpp
+void compile_mode(stencil_program *p, Mode &m);
+void load_mode(stencil_program *p, Mode &m);
+void launch(stencil_program *p, Mode &m, int i, void *stream, int chunk_first, int chunk_step,
+            int nchunks);
+void ensure_cuda();
+void unload_mode(Mode &m);
+
+// comm.cpp
+void exchange(stencil_program *p, const std::vector<int> &arrays, int depth, void *stream);
+}  // namespace sf

@@ -1,0 +1,108 @@
+"""GPU parity: the CUDA path (through the C ABI) against the CPU oracle.
+
+Bar (BASELINE north star): inf-norm relative error <= 1e-12
+(fp64) / 1e-5 (fp32) in the perf build (FMA contraction on); bit-exact against
+the oracle and between fused and unfused with fmad=0 (the parity build:
+same term order, no contraction, R4).  TEMP interiors are NaN-poisoned so a
+fused kernel consuming a value it did not compute fails loudly.
+"""
+import json
+import os
+
+import numpy as np
+import pytest
+
+from _harness import assert_close, gpu_run, oracle_outputs, rel_err
+from synth import programs as P
+
+pytestmark = pytest.mark.gpu
+
+GOLDEN = os.path.join(os.path.dirname(__file__), "golden")
+
+
+def closed_chain3_inputs(prog):
+    g = prog["grid"]
+    h = 1
+    k, j, i = np.meshgrid(np.arange(-h, g["nz"] + h), np.arange(-h, g["ny"] + h),
+                          np.arange(-h, g["nx"] + h), indexing="ij")
+    f = {"A": i + 2.0 * j + 4 * k, "B": 1.0 + 0 * i, "T1": 2 * i + 4 * j + 8 * k + 1.0,
+         "T2": 2 * i + 4 * j + 8 * k + 5.0, "O": 0.0 * i}
+    out = {}
+    for n, v in f.items():
+        v = np.ascontiguousarray(v, dtype=np.float64)
+        if n in ("T1", "T2", "O"):
+            v[h:-h, h:-h, h:-h] = np.nan
+        out[n] = v
+    return out
+
+
+@pytest.mark.parametrize("mode", ["unfused", "fused"])
+@pytest.mark.parametrize("fmad", [0, 1])
+def test_chain3_golden(cuda_device, mode, fmad):
+    prog = P.chain3()
+    gold = json.load(open(os.path.join(GOLDEN, "chain3.json")))
+    got = gpu_run(prog, mode, 0, options={"fmad": fmad}, plan=prog["plans"]["fused"],
+                  inputs=closed_chain3_inputs(prog))
+    O = got["O"]
+    for pt in gold["points"]:
+        assert O[pt["k"], pt["j"], pt["i"]] == pt["O"]
+    kk, jj, ii = np.meshgrid(np.arange(4), np.arange(4), np.arange(4), indexing="ij")
+    assert np.array_equal(O, 1.5 * ii + 3 * jj + 6 * kk + 8.25)
+
+
+CASES = [
+    # (config builder, grid override, plan names)
+    ("C1", P.c1(n=32), ["fused"]),
+    ("C1odd", P.resize(P.c1(), 37, 11, 9), ["fused"]),
+    ("C2", P.c2(nx=45, ny=37, nz=29), ["fused"]),
+    ("C3", P.c3(nx=70, ny=41, nz=33), ["fused", "fission_fused", "single"]),
+    ("C5", P.c5(nx=40, ny=23, nz=19), ["fused", "single"]),
+    ("chain3", P.resize(P.chain3(), 33, 17, 13), ["fused"]),
+]
+
+
+@pytest.mark.parametrize("name,prog,plans", CASES, ids=[c[0] for c in CASES])
+@pytest.mark.parametrize("fmad", [0, 1])
+def test_parity_vs_oracle(cuda_device, name, prog, plans, fmad):
+    ref = oracle_outputs(prog, seed=11)
+    exact = fmad == 0
+    got = gpu_run(prog, "unfused", 11, options={"fmad": fmad})
+    assert_close(prog, got, ref, exact=exact)
+    for plan in plans:
+        got = gpu_run(prog, "fused", 11, options={"fmad": fmad}, plan=prog["plans"][plan])
+        assert_close(prog, got, ref, exact=exact)
+
+
+TILES = [dict(tile_x=16, tile_y=1, zchunk=1, threads=32), dict(tile_x=32, tile_y=4, zchunk=3),
+         dict(tile_x=64, tile_y=8, zchunk=7, threads=256, prefetch=1),
+         dict(tile_x=16, tile_y=16, zchunk=64, threads=512, prefetch=3)]
+
+
+@pytest.mark.parametrize("tiles", TILES, ids=[str(i) for i in range(len(TILES))])
+def test_tile_independence_bitexact(cuda_device, tiles):
+    """Fused == unfused == oracle bit-exact with fmad=0 for any tile/chunk (P6)."""
+    for prog, plan in [(P.c2(nx=37, ny=19, nz=17), "fused"),
+                       (P.c3(nx=40, ny=21, nz=15), "fission_fused")]:
+        ref = oracle_outputs(prog, seed=5)
+        opts = dict(tiles, fmad=0)
+        got = gpu_run(prog, "fused", 5, options=opts, plan=prog["plans"][plan])
+        assert_close(prog, got, ref, exact=True)
+        got = gpu_run(prog, "unfused", 5, options=opts)
+        assert_close(prog, got, ref, exact=True)
+
+
+def test_c2_full_size(cuda_device):
+    """BASELINE configs[1] at its full size (256^3 fp64), perf build, vs the oracle."""
+    prog = P.c2()
+    ref = oracle_outputs(prog, seed=2)
+    for mode in ("unfused", "fused"):
+        got = gpu_run(prog, mode, 2, plan=prog["plans"]["fused"])
+        assert_close(prog, got, ref)
+
+
+def test_c1_fused_equals_unfused_bitexact_perf_build(cuda_device):
+    """With FMA contraction on, fused and unfused still evaluate identical expressions."""
+    prog = P.c1()
+    a = gpu_run(prog, "unfused", 1)
+    b = gpu_run(prog, "fused", 1, plan=prog["plans"]["fused"])
+    assert a["B"].tobytes() == b["B"].tobytes()

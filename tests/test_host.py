@@ -1,0 +1,249 @@
+"""Host-side logic of the library (no GPU): C-ABI exports, program validation,
+DDG/OEG edges, fission (Algorithm 2), plan legality, group analysis, the
+byte/flop model and NVRTC compilation of the generated sm_100a kernels."""
+import ctypes
+import re
+
+import pytest
+
+from paper_conf_hpdc_wahibm15_b200 import Program, StencilError
+from paper_conf_hpdc_wahibm15_b200._abi import EXPORTS, LIB_PATH
+from synth import programs as P
+
+pytestmark = pytest.mark.host
+
+HEADER = "include/stencilfuse.h"
+
+
+def test_library_exports_every_header_symbol():
+    import os
+    root = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+    text = open(os.path.join(root, HEADER)).read()
+    declared = set(re.findall(r"^\s*(?:sp_status|void|const char \*)\s*\*?\s*(\w+)\s*\(", text, re.M))
+    assert declared == set(EXPORTS), declared ^ set(EXPORTS)
+    lib = ctypes.CDLL(LIB_PATH)
+    for name in declared:
+        assert hasattr(lib, name), name
+
+
+def test_no_gpu_run_fails_loudly_without_device():
+    import torch
+    if torch.cuda.is_available():
+        pytest.skip("a GPU is present")
+    p = Program(P.c1(n=8))
+    with pytest.raises(StencilError) as e:
+        p.run_unfused(stream=0)
+    assert e.value.code in (8, 10)  # SP_E_CUDA (no device) / SP_E_STATE (unbound)
+
+
+# ----------------------------------------------------------------- validation
+def bad(prog):
+    with pytest.raises(StencilError) as e:
+        Program(prog)
+    return e.value.code
+
+
+def test_rejects_r3_in_kernel_race():
+    prog = P.c1(n=8)
+    prog["kernels"] = [P.kernel("K", P.stmt("T", [{"c": 1.0, "a": ["A", 0, 0, 0]}]),
+                                P.stmt("B", [{"c": 1.0, "a": ["T", 0, 1, 0]}]))]
+    assert bad(prog) == 2
+
+
+def test_rejects_tap_beyond_ghost():
+    prog = P.c1(n=8)
+    prog["kernels"] = [P.kernel("K", P.stmt("T", [{"c": 1.0, "a": ["A", 0, 0, 2]}]))]
+    assert bad(prog) == 2
+
+
+def test_rejects_write_to_input():
+    prog = P.c1(n=8)
+    prog["kernels"] = [P.kernel("K", P.stmt("A", [{"c": 1.0, "a": ["T", 0, 0, 0]}]))]
+    assert bad(prog) == 2
+
+
+def test_layout_alignment():
+    for prog in (P.c1(n=33), P.c3(n=17)):
+        p = Program(prog)
+        L = p.layout
+        assert (L["x_pitch"] * p.elem) % 128 == 0
+        assert (L["origin_x"] * p.elem) % 128 == 0
+        assert L["origin_x"] >= p.ghost[0] and L["x_pitch"] >= L["origin_x"] + p.n[0] + p.ghost[0]
+        assert L["bytes"] == L["x_pitch"] * L["y_alloc"] * L["z_alloc"] * p.elem
+
+
+# ----------------------------------------------------------------- DDG / OEG
+def test_edges_c2():
+    p = Program(P.c2(n=8))
+    e = {(a, b): k for a, b, k, _ in p.edges()}
+    # stmt ids: grad 0,1,2; flux 3,4,5; div 6; update 7
+    assert e[(0, 3)] & 1 and e[(1, 4)] & 1 and e[(2, 5)] & 1      # RAW g -> F
+    assert e[(3, 6)] & 1 and e[(6, 7)] & 1                         # RAW F -> D -> phin
+    assert (0, 1) not in e and (3, 4) not in e                     # independent siblings
+
+
+def test_edges_war_waw_c5_temp_reuse():
+    p = Program(P.c5(nx=8, ny=8, nz=8))
+    kinds = {}
+    for a, b, k, arr in p.edges():
+        kinds[(a, b)] = k
+    # tracer 1's gradient (stmt 8) rewrites gx (stmt 0 wrote it, stmt 3 read it)
+    assert kinds[(0, 8)] & 4          # WAW
+    assert kinds[(3, 8)] & 2          # WAR
+
+
+# ----------------------------------------------------------------- fission
+def fig3_program():
+    """Reconstruction of Fig. 3's Kern_A (garbled): R, W <- S, V and
+    T, U <- Q, P; after fission Kern_X keeps R, W with S, V."""
+    arr = [(n, "in") for n in "SVQP"] + [(n, "out") for n in "RWTU"]
+    st = lambda o, a, b: P.stmt(o, [{"c": 1.0, "a": [a, 0, 0, 0]}, {"c": 0.5, "a": [b, 1, 0, 0]}])
+    return {"name": "fig3", "dtype": "f64", "grid": {"nx": 8, "ny": 8, "nz": 8, "ghost": [1, 1, 1]},
+            "arrays": [{"name": n, "role": r} for n, r in arr],
+            "kernels": [P.kernel("Kern_A", st("R", "S", "V"), st("T", "Q", "P"), st("W", "S", "V"),
+                                 st("U", "P", "Q"))]}
+
+
+def test_fission_fig3():
+    p = Program(fig3_program())
+    comp, n = p.fission("Kern_A")
+    assert n == 2
+    assert comp == [0, 1, 0, 1]  # {R, W} and {T, U}, ordered by first statement
+
+
+def test_fission_c3_k0_separable_and_shared_input_stays():
+    p = Program(P.c3(n=8))
+    assert p.fission("K0") == ([0, 1], 2)
+    prog = P.c3(n=8)
+    prog["kernels"][0]["stmts"][1]["terms"].append({"c": 1.0, "a": ["A", 0, 0, 0]})
+    assert Program(prog).fission("K0") == ([0, 0], 1)  # shared input A joins the pieces
+
+
+# ----------------------------------------------------------------- plan legality
+def test_plan_partition_errors():
+    prog = P.c2(n=8)
+    p = Program(prog)
+    with pytest.raises(StencilError) as e:
+        p.set_plan([["grad", "flux"], ["div"]])            # update missing
+    assert e.value.code == 3
+    with pytest.raises(StencilError) as e:
+        p.set_plan([["grad", "flux"], ["flux:0", "div", "update"]])  # twice
+    assert e.value.code == 3
+
+
+def test_plan_order_error():
+    p = Program(P.c2(n=8))
+    with pytest.raises(StencilError) as e:
+        p.set_plan([["flux", "div", "update"], ["grad"]])
+    assert e.value.code == 4
+
+
+def test_plan_hazard_war_in_group():
+    """K1 reads A at +x, K2 writes A (stored for a later group): SP_E_PLAN_HAZARD (R11)."""
+    prog = {"name": "war", "dtype": "f64", "grid": {"nx": 16, "ny": 8, "nz": 8, "ghost": [1, 1, 1]},
+            "arrays": [{"name": "A", "role": "inout"}, {"name": "X", "role": "in"},
+                       {"name": "T", "role": "out"}],
+            "kernels": [P.kernel("K1", P.stmt("T", [{"c": 0.5, "a": ["A", 1, 0, 0]}])),
+                        P.kernel("K2", P.stmt("A", [{"c": 2.0, "a": ["X", 0, 0, 0]}]))]}
+    p = Program(prog)
+    with pytest.raises(StencilError) as e:
+        p.set_plan([["K1", "K2"]])
+    assert e.value.code == 5
+    p.set_plan([["K1"], ["K2"]])  # split: legal
+    # point-wise read of the own tile before the store is the allowed exception
+    prog["kernels"][0]["stmts"][0]["terms"][0]["a"] = ["A", 0, 0, 0]
+    Program(prog).set_plan([["K1", "K2"]])
+
+
+def test_failed_plan_keeps_previous():
+    p = Program(P.c2(n=8))
+    p.set_plan([["grad", "flux", "div", "update"]])
+    with pytest.raises(StencilError):
+        p.set_plan([["update"], ["grad", "flux", "div"]])
+    assert p.n_launches("fused") == 1
+
+
+# ----------------------------------------------------------------- analysis / model
+def passes(p, mode):
+    return sum(r["bytes_alg"] for r in p.reports(mode)) / p.elem
+
+
+def test_bytes_model_c2():
+    """C2: unfused 21 passes -> fused 5 (pin P10)."""
+    prog = P.c2(n=64)
+    p = Program(prog)
+    assert passes(p, "unfused") == 21
+    p.set_plan(prog["plans"]["fused"])
+    assert passes(p, "fused") == 5
+    r = p.reports("fused")[0]
+    assert r["n_inputs"] == 4 and r["n_stores"] == 1
+
+
+def test_bytes_model_c3():
+    """C3: 21 -> 8 (no fission) -> 5 (fission + fusion) -> 3 (single group)."""
+    prog = P.c3(n=64)
+    p = Program(prog)
+    assert passes(p, "unfused") == 21
+    for plan, want in (("fused", 8), ("fission_fused", 5), ("single", 3)):
+        p.set_plan(prog["plans"][plan])
+        assert passes(p, "fused") == want, plan
+
+
+def test_group_analysis_c2_appendix_b():
+    """Per-statement extension/lead/storage of C2's fused group."""
+    prog = P.c2(n=64)
+    p = Program(prog)
+    p.set_plan(prog["plans"]["fused"])
+    src = p.source("fused")
+    info = {}
+    for m in re.finditer(r"// stmt (\S+) -> (\S+)\s+lead (-?\d+), planes \[(-?\d+), zc-1\+(-?\d+)\], "
+                         r"ext \((-?\d+),(-?\d+),(-?\d+),(-?\d+)\)(, stored)?, (register|smem ring) "
+                         r"depth (\d+)", src):
+        info[m.group(2)] = dict(lead=int(m.group(3)), ext=tuple(int(m.group(i)) for i in range(6, 10)),
+                                stored=bool(m.group(10)), keep=m.group(11), depth=int(m.group(12)))
+    assert info["phin"] == dict(lead=0, ext=(0, 0, 0, 0), stored=True, keep="register", depth=1)
+    assert info["D"]["ext"] == (0, 0, 0, 0) and info["D"]["keep"] == "register"
+    assert info["Fx"]["ext"] == (1, 1, 0, 0) and info["Fx"]["keep"] == "smem ring"
+    assert info["Fy"]["ext"] == (0, 0, 1, 1) and info["Fy"]["keep"] == "smem ring"
+    assert info["Fz"] == dict(lead=1, ext=(0, 0, 0, 0), stored=False, keep="register", depth=3)
+    assert info["gx"]["ext"] == (1, 1, 0, 0) and info["gx"]["keep"] == "register"
+    assert info["gz"]["lead"] == 1 and info["gz"]["keep"] == "register"
+
+
+def test_group_analysis_chain3():
+    prog = P.chain3()
+    p = Program(prog)
+    p.set_plan(prog["plans"]["fused"])
+    src = p.source("fused")
+    assert re.search(r"-> T2\s+lead 1, planes \[0, zc-1\+1\], ext \(1,0,0,0\)", src)
+    assert re.search(r"-> T1\s+lead 1, planes \[0, zc-1\+1\], ext \(1,0,1,0\)", src)
+
+
+def test_dead_statement_skipped():
+    """A TEMP overwritten before any read inside the group is never computed."""
+    prog = {"name": "dead", "dtype": "f64", "grid": {"nx": 16, "ny": 8, "nz": 8, "ghost": [1, 1, 1]},
+            "arrays": [{"name": "X", "role": "in"}, {"name": "T", "role": "temp"},
+                       {"name": "Y", "role": "out"}],
+            "kernels": [P.kernel("K1", P.stmt("T", [{"c": 3.0, "a": ["X", 1, 0, 0]}])),
+                        P.kernel("K2", P.stmt("T", [{"c": 2.0, "a": ["X", 0, 0, 0]}])),
+                        P.kernel("K3", P.stmt("Y", [{"c": 1.0, "a": ["T", 0, 0, 1]}]))]}
+    p = Program(prog)
+    p.set_plan([["K1", "K2", "K3"]])
+    assert p.reports("fused")[0]["n_stmts"] == 2
+
+
+# ----------------------------------------------------------------- NVRTC (sm_100a) compile
+@pytest.mark.parametrize("name", ["C1", "C2", "C3", "C5", "chain3"])
+def test_generated_kernels_compile_for_sm100a(name):
+    prog = P.chain3() if name == "chain3" else P.CONFIGS[name]()
+    for fmad in (0, 1):
+        p = Program(prog, options={"fmad": fmad})
+        p.compile("unfused")
+        for plan_name, plan in prog["plans"].items():
+            if plan_name == "unfused":
+                continue
+            p.set_plan(plan)
+            p.compile("fused")
+            for r in p.reports("fused"):
+                assert 0 < r["regs_per_thread"] <= 255
+                assert r["smem_bytes"] <= 227 * 1024

@@ -1,0 +1,383 @@
+"""Benchmark of the fused stencil-DAG executor (driver contract).
+
+  python bench.py [--gpus N] [--steps K] [--warmup W] [--workload C4] [--impl ours|reference]
+
+One step = one pass of the whole hot path over the workload: every group of the
+fusion plan, in plan order (run_fused), plus on N > 1 ranks the z-slab halo
+exchanges.  Metric (BASELINE.json): grid-point updates/s (interior points x
+original kernels / s, reading R21) and HBM GB/s against the roofline, fused vs
+unfused.  N > 1: one process per GPU (torchrun), z-slab decomposition, weak
+scaling (per-GPU grid fixed).  Inputs: seeded synthetic fields (synth/), 2.1 GB
+per GPU for C4 (larger than the 126 MB L2, so no flush between steps).
+
+--impl reference times the CPU oracle (oracle/, the plain serial program) on a
+bounded sample of the same workload, as the reference arm.
+"""
+from __future__ import annotations
+
+import argparse
+import json
+import os
+import statistics
+import subprocess
+import sys
+import threading
+import time
+
+ROOT = os.path.dirname(os.path.abspath(__file__))
+sys.path.insert(0, ROOT)
+
+METRIC = "grid-point updates/s and HBM GB/s (% of roofline), fused vs unfused, 1/2/4/8 B200"
+UNIT = "grid-point updates/s"
+
+
+def load_workload(name):
+    from synth import programs as P
+    if name == "C4":
+        from synth.scale_les import c4
+        prog = c4()
+        plan_path = os.path.join(ROOT, "configs", "c4_plan.json")
+        if os.path.exists(plan_path):
+            prog["plans"]["fused"] = json.load(open(plan_path))["groups"]
+        return prog
+    return P.CONFIGS[name]()
+
+
+def plan_of(prog):
+    if "fused" in prog["plans"]:
+        return prog["plans"]["fused"]
+    from paper_conf_hpdc_wahibm15_b200 import Program
+    return Program(prog).plan_greedy()
+
+
+def peaks():
+    try:
+        return json.load(open(os.path.join(ROOT, "MEASURED_PEAKS.json")))
+    except Exception:
+        return None
+
+
+class ClockSampler:
+    """nvidia-smi clocks / throttle reasons sampled during the timed region."""
+
+    FIELDS = ("clocks.sm,clocks.max.sm,clocks_event_reasons.hw_slowdown,"
+              "clocks_event_reasons.hw_thermal_slowdown,clocks_event_reasons.sw_thermal_slowdown,"
+              "clocks_event_reasons.sw_power_cap")
+
+    def __init__(self, device_index):
+        self.idx = device_index
+        self.proc = None
+        self.lines = []
+
+    def start(self):
+        try:
+            self.proc = subprocess.Popen(
+                ["nvidia-smi", "-i", str(self.idx), f"--query-gpu={self.FIELDS}",
+                 "--format=csv,noheader,nounits", "-lms", "100"],
+                stdout=subprocess.PIPE, stderr=subprocess.DEVNULL, text=True)
+            self.t = threading.Thread(target=self._read, daemon=True)
+            self.t.start()
+        except Exception:
+            self.proc = None
+
+    def _read(self):
+        for line in self.proc.stdout:
+            self.lines.append(line.strip())
+
+    def stop(self):
+        if not self.proc:
+            return {"sm_mhz": None, "sm_max_mhz": None, "reasons": ["nvidia-smi unavailable"]}
+        self.proc.terminate()
+        try:
+            self.proc.wait(timeout=5)
+        except Exception:
+            self.proc.kill()
+        sm, mx, reasons = [], [], set()
+        names = ["hw_slowdown", "hw_thermal_slowdown", "sw_thermal_slowdown", "sw_power_cap"]
+        for ln in self.lines:
+            parts = [x.strip() for x in ln.split(",")]
+            if len(parts) < 6:
+                continue
+            try:
+                sm.append(float(parts[0]))
+                mx.append(float(parts[1]))
+            except ValueError:
+                continue
+            for n, v in zip(names, parts[2:]):
+                if v.lower().startswith("active"):
+                    reasons.add(n)
+        return {"sm_mhz": statistics.median(sm) if sm else None,
+                "sm_max_mhz": max(mx) if mx else None, "reasons": sorted(reasons),
+                "samples": len(sm)}
+
+
+def fill_inputs(p, prog, device, z_offset, zhalo):
+    from synth.fields import field_torch
+    hz = p.ghost[2]
+    extra = (zhalo - hz, zhalo - hz)
+    for aid, a in enumerate(prog["arrays"]):
+        v = field_torch(4, aid, p.n, p.ghost, prog["dtype"], device, z_offset=z_offset,
+                        nz_alloc_extra=extra)
+        p.padded_view(p.tensors[a["name"]], hz=zhalo).copy_(v)
+
+
+def run_ours(args):
+    import torch
+    import torch.distributed as dist
+
+    from paper_conf_hpdc_wahibm15_b200 import Comm, Program
+
+    world = int(os.environ.get("WORLD_SIZE", "1"))
+    rank = int(os.environ.get("RANK", "0"))
+    local = int(os.environ.get("LOCAL_RANK", "0"))
+    if world > 1:
+        torch.cuda.set_device(local)
+        dist.init_process_group("nccl", device_id=torch.device("cuda", local))
+    dev = torch.device("cuda", local if world > 1 else 0)
+    torch.cuda.set_device(dev)
+    prog = load_workload(args.workload)
+    plan = plan_of(prog)
+    nz = prog["grid"]["nz"]
+    # deep halo needed by the plan's accumulated z-reach (probe on the local grid)
+    probe = Program(prog)
+    probe.set_plan(plan)
+    reach = max([max(r["z_below"], r["z_above"]) for r in probe.reports("fused")] + [prog["grid"]["ghost"][2]])
+    zhalo = reach if world > 1 else prog["grid"]["ghost"][2]
+    del probe
+    comm = Comm(rank, world) if world > 1 else None
+    p = Program(prog, comm=comm, nz_global=nz * world, z_offset=rank * nz, zhalo=zhalo)
+    p.set_plan(plan)
+    p.allocate(dev, fill=0.0)
+    fill_inputs(p, prog, dev, rank * nz, zhalo)
+    stream = torch.cuda.current_stream(dev)
+    n_pts = prog["grid"]["nx"] * prog["grid"]["ny"] * nz  # per GPU
+    n_kernels = len(prog["kernels"])
+    reps_f = p.reports("fused")
+    reps_u = p.reports("unfused")
+    live_f = [i for i, r in enumerate(reps_f) if r["grid_ctas"] > 0]
+
+    def barrier():
+        if world > 1:
+            dist.barrier()
+        torch.cuda.synchronize(dev)
+
+    def max_over_ranks(x):
+        if world == 1:
+            return x
+        t = torch.tensor([x], dtype=torch.float64, device=dev)
+        dist.all_reduce(t, op=dist.ReduceOp.MAX)
+        return float(t.item())
+
+    # ---------------------------------------------------------- fused, timed
+    for _ in range(args.warmup):
+        p.run_fused(stream)
+    barrier()
+    sampler = ClockSampler(dev.index)
+    sampler.start()
+    time.sleep(0.25)
+    per_launch = [0.0] * len(reps_f)
+    if world == 1:
+        # events between launches: per-launch durations on the launching stream
+        evs = [[torch.cuda.Event(enable_timing=True) for _ in range(len(live_f) + 1)]
+               for _ in range(args.steps)]
+        barrier()
+        t0 = time.perf_counter()
+        for k in range(args.steps):
+            for j, i in enumerate(live_f):
+                evs[k][j].record(stream)
+                p.run_launch("fused", i, stream)
+            evs[k][-1].record(stream)
+        barrier()
+        wall = time.perf_counter() - t0
+        step_ms = sum(evs[k][0].elapsed_time(evs[k][-1]) for k in range(args.steps)) / args.steps
+        for j, i in enumerate(live_f):
+            per_launch[i] = sum(evs[k][j].elapsed_time(evs[k][j + 1])
+                                for k in range(args.steps)) / args.steps
+    else:
+        s, e = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+        barrier()
+        t0 = time.perf_counter()
+        s.record(stream)
+        for k in range(args.steps):
+            p.run_fused(stream)
+        e.record(stream)
+        barrier()
+        wall = time.perf_counter() - t0
+        step_ms = s.elapsed_time(e) / args.steps
+    clocks = sampler.stop()
+    step_ms = max_over_ranks(step_ms)
+    if world > 1:  # per-launch durations from a separate pass (no exchange)
+        for i in live_f:
+            s, e = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+            s.record(stream)
+            for _ in range(10):
+                p.run_launch("fused", i, stream)
+            e.record(stream)
+            torch.cuda.synchronize(dev)
+            per_launch[i] = s.elapsed_time(e) / 10
+
+    # ---------------------------------------------------------- unfused, same K
+    for _ in range(args.warmup):
+        p.run_unfused(stream)
+    s, e = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+    barrier()
+    s.record(stream)
+    for _ in range(args.steps):
+        p.run_unfused(stream)
+    e.record(stream)
+    barrier()
+    unf_ms = max_over_ranks(s.elapsed_time(e) / args.steps)
+
+    # ---------------------------------------------------------- e2e through the public API
+    in_names = [a["name"] for a in prog["arrays"] if a["role"] in ("in", "inout")]
+    out_names = [a["name"] for a in prog["arrays"] if a["role"] in ("out", "inout")]
+    host_in = {n: torch.empty_like(p.tensors[n], device="cpu").pin_memory() for n in in_names}
+    host_out = {n: torch.empty_like(p.tensors[n], device="cpu").pin_memory() for n in out_names}
+    for n in in_names:
+        host_in[n].copy_(p.tensors[n])
+    e2e_steps = max(1, min(args.steps, 10))
+    barrier()
+    s, e = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+    s.record(stream)
+    for _ in range(e2e_steps):
+        for n in in_names:
+            p.tensors[n].copy_(host_in[n], non_blocking=True)
+        p.run_fused(stream)
+        for n in out_names:
+            host_out[n].copy_(p.tensors[n], non_blocking=True)
+    e.record(stream)
+    barrier()
+    e2e_ms = max_over_ranks(s.elapsed_time(e) / e2e_steps)
+    h2d = sum(host_in[n].numel() * host_in[n].element_size() for n in in_names)
+    d2h = sum(host_out[n].numel() * host_out[n].element_size() for n in out_names)
+
+    # ---------------------------------------------------------- report (rank 0)
+    if rank == 0:
+        pk = peaks()
+        peak = pk["hbm_gbs"] if pk else 6650.0
+        peak_src = "MEASURED_PEAKS.json hbm_gbs (measured copy)" if pk else "fallback 6.65 TB/s"
+        updates = n_pts * world * n_kernels
+        value = updates / (step_ms * 1e-3)
+        # dominant kernel: largest share of the step
+        dom = max(live_f, key=lambda i: per_launch[i])
+        r = reps_f[dom]
+        achieved = r["bytes_alg"] * n_pts / (per_launch[dom] * 1e-3) / 1e9
+        traffic = None
+        tp = os.path.join(ROOT, "profiles", f"ncu_traffic_{args.workload}.json")
+        if os.path.exists(tp):
+            traffic = json.load(open(tp)).get(f"sf_fused_{dom}")
+        alg_step = sum(x["bytes_alg"] for x in reps_f) * n_pts
+        alg_step_u = sum(x["bytes_alg"] for x in reps_u) * n_pts
+        line = {
+            "metric": METRIC, "value": value, "unit": UNIT, "n_gpus": world,
+            "steps": args.steps, "warmup": args.warmup, "ms_per_step": step_ms,
+            "higher_is_better": True, "scaling": "weak", "vs_baseline": None,
+            "dtype": prog["dtype"], "data": "synthetic: seeded splitmix64 uniform[-1,1) fields",
+            "config": {"workload": args.workload, "grid_per_gpu": [prog["grid"]["nx"], prog["grid"]["ny"], nz],
+                       "kernels": n_kernels, "arrays": len(prog["arrays"]),
+                       "fused_groups": len(live_f), "parallelism": f"z-slab x{world}",
+                       "l2": "no flush: per-GPU working set > 126 MB L2"},
+            "hbm_gbs_alg": alg_step / (step_ms * 1e-3) / 1e9,
+            "roofline_step": {"achieved": alg_step / (step_ms * 1e-3) / 1e9, "peak": peak,
+                              "unit": "GB/s", "frac": alg_step / (step_ms * 1e-3) / 1e9 / peak,
+                              "frac_of_8tbs_nominal": alg_step / (step_ms * 1e-3) / 8e12},
+            "roofline": {"bound": "hbm", "achieved": achieved, "peak": peak, "unit": "GB/s",
+                         "frac": achieved / peak, "traffic": traffic, "kernel": f"sf_fused_{dom}",
+                         "share_of_step": per_launch[dom] / step_ms, "peak_source": peak_src},
+            "fused_vs_unfused": {"unfused_ms_per_step": unf_ms,
+                                 "unfused_value": updates / (unf_ms * 1e-3),
+                                 "speedup": unf_ms / step_ms,
+                                 "bytes_alg_per_step": {"fused": alg_step, "unfused": alg_step_u},
+                                 "predicted_traffic_reduction": 1 - alg_step / alg_step_u},
+            "e2e": {"value": updates / (e2e_ms * 1e-3), "unit": UNIT, "h2d_bytes_per_step": h2d,
+                    "d2h_bytes_per_step": d2h, "ms_per_step": e2e_ms},
+            "gpu_launches": args.steps * len(live_f),
+            "clocks": clocks,
+            "wall_s_timed": wall,
+        }
+        if world == 1 and not args.no_cpu:
+            line["cpu_baseline"] = cpu_baseline(args, budget_s=15.0)
+        print(json.dumps(line), flush=True)
+    if world > 1:
+        dist.barrier()
+        dist.destroy_process_group()
+
+
+def oracle_step_time(prog, nz_s, seed=4):
+    from oracle import OracleProgram, dense_arrays
+    from synth.programs import resize
+    g = prog["grid"]
+    sub = resize(prog, g["nx"], g["ny"], nz_s)
+    arrs = dense_arrays(sub, seed)
+    o = OracleProgram(sub)
+    t0 = time.perf_counter()
+    o.run(arrs)
+    return time.perf_counter() - t0, sub
+
+
+def cpu_baseline(args, budget_s=15.0, steps=1):
+    """The oracle (single thread, as it stands) on a z-subslab of the workload."""
+    prog = load_workload(args.workload)
+    g = prog["grid"]
+    t1, _ = oracle_step_time(prog, 1)
+    per_plane = max(t1, 1e-4)
+    nz_s = int(max(1, min(g["nz"], budget_s / per_plane / max(steps, 1))))
+    ts = []
+    for _ in range(steps):
+        t, sub = oracle_step_time(prog, nz_s)
+        ts.append(t)
+    t = sum(ts) / len(ts)
+    upd = g["nx"] * g["ny"] * nz_s * len(prog["kernels"])
+    return {"value": upd / t, "unit": UNIT, "cores": 1, "kind": "oracle",
+            "sample": f"{args.workload} program on a {g['nx']}x{g['ny']}x{nz_s} z-subslab, one step, "
+                      f"serial C oracle (-O2 -ffp-contract=off), {t:.2f} s"}
+
+
+def run_reference(args):
+    world = int(os.environ.get("WORLD_SIZE", "1"))
+    rank = int(os.environ.get("RANK", "0"))
+    if rank != 0:
+        return
+    prog = load_workload(args.workload)
+    g = prog["grid"]
+    t1, _ = oracle_step_time(prog, 1)
+    budget = 150.0 / max(args.steps + args.warmup, 1)
+    nz_s = int(max(1, min(g["nz"], budget / max(t1, 1e-4))))
+    for _ in range(args.warmup):
+        oracle_step_time(prog, nz_s)
+    ts = [oracle_step_time(prog, nz_s)[0] for _ in range(args.steps)]
+    t = sum(ts) / len(ts)
+    upd = g["nx"] * g["ny"] * nz_s * len(prog["kernels"])
+    v = upd / t
+    sample = (f"{args.workload} program on a {g['nx']}x{g['ny']}x{nz_s} z-subslab per step, "
+              f"serial C oracle, 1 thread")
+    print(json.dumps({
+        "impl": "reference", "metric": METRIC, "value": v, "unit": UNIT, "n_gpus": world,
+        "steps": args.steps, "warmup": args.warmup, "ms_per_step": t * 1e3,
+        "higher_is_better": True, "scaling": "weak", "vs_baseline": None, "dtype": prog["dtype"],
+        "data": "synthetic", "config": {"workload": args.workload,
+                                        "grid_per_gpu": [g["nx"], g["ny"], g["nz"]]},
+        "cpu_baseline": {"value": v, "unit": UNIT, "cores": 1, "kind": "oracle", "sample": sample},
+        "e2e": {"value": v, "unit": UNIT, "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0},
+    }), flush=True)
+
+
+def main():
+    ap = argparse.ArgumentParser()
+    ap.add_argument("--gpus", type=int, default=1)
+    ap.add_argument("--steps", type=int, default=500)
+    ap.add_argument("--warmup", type=int, default=10)
+    ap.add_argument("--workload", default="C4", choices=["C1", "C2", "C3", "C4", "C5"])
+    ap.add_argument("--impl", default="ours", choices=["ours", "reference"])
+    ap.add_argument("--no-cpu", action="store_true", help="skip the cpu_baseline leg")
+    args = ap.parse_args()
+    if args.warmup < 3:
+        args.warmup = 3
+    if args.impl == "reference":
+        run_reference(args)
+    else:
+        run_ours(args)
+
+
+if __name__ == "__main__":
+    main()

@@ -184,6 +184,14 @@ sp_status sp_fission_components(const stencil_program *prog, int32_t kernel, int
 sp_status fusion_plan_set(stencil_program *prog, int32_t n_groups, const int32_t *group_begin,
                           const sp_stmt_ref *members);
 
+/* Greedy host-side plan search (the paper's search step, §3.2.4, with this
+ * library's byte/flop/issue model as the objective): starts from fully fissioned
+ * kernels (§4.1) and merges adjacent groups while the modelled time drops.
+ * Writes at most cap groups: group_begin[cap+1], members[number of statements].
+ * With group_begin == NULL only *n_groups is returned.  Does not set the plan. */
+sp_status sp_plan_greedy(stencil_program *prog, int32_t cap, int32_t *n_groups,
+                         int32_t *group_begin, sp_stmt_ref *members);
+
 /* mode 0 = unfused (one launch per original kernel), 1 = fused plan. */
 sp_status sp_plan_count(const stencil_program *prog, int32_t mode, int32_t *n_launches);
 sp_status sp_plan_report(const stencil_program *prog, int32_t mode, int32_t launch,

@@ -218,6 +218,18 @@ class Program:
         m = (SpStmtRef * len(members))(*[SpStmtRef(k, s) for k, s in members])
         _check(lib().fusion_plan_set(self.handle, len(groups), b, m))
 
+    def plan_greedy(self):
+        """Greedy fission/fusion plan from the library's model; list of groups of 'K:i' refs."""
+        ng = ctypes.c_int32()
+        _check(lib().sp_plan_greedy(self.handle, 0, ctypes.byref(ng), None, None))
+        nst = sum(len(k["stmts"]) for k in self.prog["kernels"])
+        begin = (ctypes.c_int32 * (ng.value + 1))()
+        mem = (SpStmtRef * nst)()
+        _check(lib().sp_plan_greedy(self.handle, ng.value, ctypes.byref(ng), begin, mem))
+        names = [k["name"] for k in self.prog["kernels"]]
+        return [[f"{names[mem[i].kernel]}:{mem[i].stmt}" for i in range(begin[g], begin[g + 1])]
+                for g in range(ng.value)]
+
     def n_launches(self, mode):
         n = ctypes.c_int32()
         _check(lib().sp_plan_count(self.handle, self._mode(mode), ctypes.byref(n)))

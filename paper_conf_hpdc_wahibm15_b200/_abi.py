@@ -74,7 +74,7 @@ EXPORTS = [
     "sp_comm_unique_id", "sp_comm_create", "sp_comm_destroy", "stencil_program_create",
     "stencil_program_destroy", "stencil_program_layout", "stencil_program_bind",
     "sp_program_set_option", "sp_program_counts", "sp_program_edges", "sp_fission_components",
-    "fusion_plan_set", "sp_plan_count", "sp_plan_report", "fusion_plan_report", "sp_plan_source",
+    "fusion_plan_set", "sp_plan_greedy", "sp_plan_count", "sp_plan_report", "fusion_plan_report", "sp_plan_source",
     "sp_compile", "run_unfused", "run_fused", "sp_run_launch", "exchange_halos", "sp_last_error",
 ]
 
@@ -102,6 +102,7 @@ def lib():
             "sp_fission_components": [vp, i32, P(i32), P(i32)],
             "fusion_plan_set": [vp, i32, P(i32), P(SpStmtRef)],
             "sp_plan_count": [vp, i32, P(i32)],
+            "sp_plan_greedy": [vp, i32, P(i32), P(i32), P(SpStmtRef)],
             "sp_plan_report": [vp, i32, i32, P(SpGroupReport)],
             "fusion_plan_report": [vp, i32, P(SpGroupReport)],
             "sp_plan_source": [vp, i32, ctypes.c_char_p, ctypes.c_size_t, P(ctypes.c_size_t)],

@@ -49,6 +49,16 @@ __device__ __forceinline__ void sf_mbar_wait(sf_u64 *bar, sf_u32 parity) {
         : "memory");
 }
 
+// consumer release of a ring slot (default .release.cta semantics)
+__device__ __forceinline__ void sf_mbar_arrive(sf_u64 *bar) {
+    asm volatile("mbarrier.arrive.shared::cta.b64 _, [%0];" ::"r"(sf_smem_addr(bar)) : "memory");
+}
+
+// named barrier over the compute warps only (the producer warp never joins)
+__device__ __forceinline__ void sf_bar_sync(int id, int nthreads) {
+    asm volatile("bar.sync %0, %1;" ::"r"(id), "r"(nthreads) : "memory");
+}
+
 __device__ __forceinline__ void sf_prefetch_tmap(const SfTmap *m) {
     asm volatile("prefetch.tensormap [%0];" ::"l"(m) : "memory");
 }
@@ -70,6 +80,20 @@ __device__ __forceinline__ void sf_st(double *p, double v) {
 }
 __device__ __forceinline__ void sf_st(float *p, float v) {
     asm volatile("st.global.L1::no_allocate.f32 [%0], %1;" ::"l"(p), "f"(v) : "memory");
+}
+// ghost value of a point outside the global interior: predicated non-coherent
+// load (ghost cells are never written), 0 when the point is outside the allocation
+__device__ __forceinline__ double sf_ldg_pred(const double *p, bool pred) {
+    double v = 0.0;
+    asm("{\n\t.reg .pred P1;\n\tsetp.ne.b32 P1, %2, 0;\n\t@P1 ld.global.nc.f64 %0, [%1];\n}"
+        : "+d"(v) : "l"(p), "r"((int)pred));
+    return v;
+}
+__device__ __forceinline__ float sf_ldg_pred(const float *p, bool pred) {
+    float v = 0.0f;
+    asm("{\n\t.reg .pred P1;\n\tsetp.ne.b32 P1, %2, 0;\n\t@P1 ld.global.nc.f32 %0, [%1];\n}"
+        : "+f"(v) : "l"(p), "r"((int)pred));
+    return v;
 }
 __device__ __forceinline__ double sf_ld(const double *p) {
     double v;

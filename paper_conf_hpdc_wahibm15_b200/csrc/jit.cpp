@@ -263,7 +263,7 @@ void launch(stencil_program *p, Mode &m, int i, void *stream, int chunk_first, i
     std::memcpy(base + L.int_off, ints, 8);
     void *args[] = {base};
     drv_check(g_drv.LaunchKernel((CUfunction)L.func, (unsigned)L.ntx, (unsigned)L.nty,
-                                 (unsigned)nchunks, (unsigned)L.nt, 1, 1, (unsigned)L.smem,
+                                 (unsigned)nchunks, (unsigned)L.nth, 1, 1, (unsigned)L.smem,
                                  (CUstream)stream, args, nullptr),
               "cuLaunchKernel");
 }

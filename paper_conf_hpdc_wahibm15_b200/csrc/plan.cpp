@@ -79,7 +79,9 @@ static Launch analyze_group(const stencil_program *p, const std::vector<int> &me
         }
         if (!A.any) continue;  // dead: nothing consumes it
         G.needed = true;
-        G.ex0 = A.ex0; G.ex1 = A.ex1; G.ey0 = A.ey0; G.ey1 = A.ey1;
+        // every region contains the tile core (the shared thread mapping of the core)
+        G.ex0 = std::max(A.ex0, 0); G.ex1 = std::max(A.ex1, 0);
+        G.ey0 = std::max(A.ey0, 0); G.ey1 = std::max(A.ey1, 0);
         G.loff = A.loff; G.lead = A.lead;
         G.depth = G.lead - std::min(A.minread, G.lead) + 1;
         for (const TermR &t : G.terms) {
@@ -209,12 +211,18 @@ static Launch analyze_group(const stencil_program *p, const std::vector<int> &me
 // -------------------------------------------------------- config and model
 struct Cost { double t; int64_t smem; };
 
+static int pow2ceil(int v) {
+    int r = 1;
+    while (r < v) r <<= 1;
+    return r;
+}
+
 static void layout_launch(const stencil_program *p, Launch &L) {
     if (L.tx % (16 / p->elem)) fail(SP_E_ARG, "tile_x must be a multiple of 16 bytes");
     const int e = p->elem;
     L.rw_pad = 16 / e;  // TMA: inner box extent multiple of 16 B
-    L.in_off.clear(); L.in_plane.clear(); L.in_rw.clear(); L.in_rh.clear();
-    L.st_off.clear(); L.st_plane.clear(); L.st_w.clear(); L.st_h.clear();
+    L.in_off.clear(); L.in_plane.clear(); L.in_rw.clear(); L.in_rh.clear(); L.in_depth.clear();
+    L.st_off.clear(); L.st_plane.clear(); L.st_w.clear(); L.st_h.clear(); L.st_depth.clear();
     int64_t off = 0;
     L.n_bars = 0;
     for (Input &I : L.in) {
@@ -224,32 +232,98 @@ static void layout_launch(const stencil_program *p, Launch &L) {
         int rw = (int)rup(L.tx + I.bx0 + std::max(I.ex1, 0), L.rw_pad);
         int rh = L.ty + I.ey0 + I.ey1;
         int64_t plane = rup((int64_t)rw * rh, 128 / e);
-        int D = I.ahi - I.alo + 1 + L.pf;
+        int D = pow2ceil(I.ahi - I.alo + 1 + L.pf);
         L.in_off.push_back(off);
         L.in_plane.push_back(plane);
         L.in_rw.push_back(rw);
         L.in_rh.push_back(rh);
+        L.in_depth.push_back(D);
         off += plane * D * e;
-        L.n_bars += D;
     }
+    L.nbar_full = pow2ceil(L.pf + 1);
+    L.nbar_empty = pow2ceil(L.pf + 2);
+    L.n_bars = L.nbar_full + L.nbar_empty;
     for (const Stage &G : L.st) {
         int w = L.tx + G.ex0 + G.ex1, h = L.ty + G.ey0 + G.ey1;
         L.st_w.push_back(w);
         L.st_h.push_back(h);
         if (G.keep == Keep::Smem) {
+            // one plane deeper than the reuse distance: no end-of-step barrier needed
+            int D = pow2ceil(G.depth + 1);
             int64_t plane = rup((int64_t)w * h, 128 / e);
             L.st_off.push_back(off);
             L.st_plane.push_back(plane);
-            off += plane * G.depth * e;
+            L.st_depth.push_back(D);
+            off += plane * D * e;
         } else {
             L.st_off.push_back(-1);
             L.st_plane.push_back(0);
+            L.st_depth.push_back(0);
         }
     }
     off = rup(off, 8);
     L.bar_off = off;
     off += 8 * (int64_t)L.n_bars;
     L.smem = rup(off, 128);
+}
+
+// register estimate of a configured launch (occupancy model of the tile chooser;
+// the paper tunes block size with the occupancy-calculator equations, §4.2)
+static int estimate_regs(const stencil_program *p, const Launch &L) {
+    const int w64 = p->elem / 4;
+    int xt, yt, cpx, cpy;
+    core_geometry(L, &xt, &yt, &cpx, &cpy);
+    const int cp = cpx * cpy;
+    std::vector<std::set<int>> lays(L.cls.size());
+    std::set<int> all;
+    std::set<std::pair<int, int>> bases;
+    for (size_t m = 0; m < L.st.size(); ++m) {
+        const Stage &G = L.st[m];
+        if (!G.needed) continue;
+        if (G.keep == Keep::Smem) { lays[G.cls].insert(1000 + (int)m); bases.insert({1000 + (int)m, G.lead}); }
+        for (const TermR &t : G.terms)
+            for (int w = 0; w < 2; ++w) {
+                if (w == 1 && !t.has_b) continue;
+                const Src &s = w ? t.b : t.a;
+                if (!s.stage) { lays[G.cls].insert(s.idx); bases.insert({s.idx, G.lead + s.dz}); }
+                else if (L.st[s.idx].keep == Keep::Smem) {
+                    lays[G.cls].insert(1000 + s.idx);
+                    bases.insert({1000 + s.idx, G.lead + s.dz});
+                }
+            }
+    }
+    for (auto &st : lays) all.insert(st.begin(), st.end());
+    int regs = 40 + (int)all.size() + (int)bases.size();
+    std::vector<int> hp(L.cls.size());
+    for (size_t c = 0; c < L.cls.size(); ++c) {
+        const RegionClass &R = L.cls[c];
+        int nh = (L.tx + R.x1 - R.x0) * (L.ty + R.y1 - R.y0) - L.tx * L.ty;
+        hp[c] = (nh + L.nt - 1) / L.nt;
+        regs += hp[c] * (2 + (int)lays[c].size());
+    }
+    for (const Stage &G : L.st)
+        if (G.keep == Keep::Reg) regs += (cp + hp[G.cls]) * G.depth * w64;
+    regs += 3 * cp * w64;
+    return regs;
+}
+
+// issued instructions per output point (thread-level), for the issue-rate ceiling
+static double estimate_instr(const Launch &L) {
+    int xt, yt, cpx, cpy;
+    core_geometry(L, &xt, &yt, &cpx, &cpy);
+    const double tile = (double)L.tx * L.ty;
+    double per_pt = 0, per_step = 60;
+    for (const Stage &G : L.st) {
+        if (!G.needed) continue;
+        double pts = (double)(L.tx + G.ex0 + G.ex1) * (L.ty + G.ey0 + G.ey1);
+        double halo = pts - tile;
+        int ops = 0;
+        for (const TermR &t : G.terms) ops += 2 + (t.has_b ? 2 : 0);
+        per_pt += (ops + 2) * 1.0 + (G.stored ? 1 : 0) + halo / tile * (ops + 10);
+        per_step += 12 + 4.0 * G.terms.size() / 2;
+    }
+    // per-step work is shared by the cp points of a thread
+    return per_pt + per_step / (cpx * cpy) * ((double)L.nt * cpx * cpy / tile);
 }
 
 // per-point byte/flop model of a configured launch
@@ -299,20 +373,24 @@ static int max_region_points(const Launch &L) {
     return m;
 }
 
-static void choose_config(const stencil_program *p, Launch &L) {
+static void choose_config(const stencil_program *p, Launch &L, bool quick = false) {
     const sp_grid &g = p->grid;
     const int e = p->elem;
     const int64_t nz = g.nz_local;
     std::vector<int> cx, cy, cz, cn, cp;
     if (p->opt.tile_x) cx = {p->opt.tile_x};
+    else if (quick) cx = e == 8 ? std::vector<int>{32, 64} : std::vector<int>{64, 128};
     else cx = e == 8 ? std::vector<int>{16, 32, 64} : std::vector<int>{32, 64, 128};
     if (p->opt.tile_y) cy = {p->opt.tile_y};
+    else if (quick) cy = {8, 16, 32};
     else cy = {1, 2, 4, 8, 16, 32};
     if (p->opt.zchunk) cz = {p->opt.zchunk};
+    else if (quick) cz = {16, 32, 64};
     else cz = {4, 8, 16, 32, 64, 128, 256, 512};
     if (p->opt.threads) cn = {p->opt.threads};
-    else cn = {128, 256, 512};
+    else cn = {64, 128, 256};
     if (p->opt.prefetch >= 0) cp = {p->opt.prefetch};
+    else if (quick) cp = {1, 2};
     else cp = {1, 2, 3};
     const double sms = p->num_sms;
     const double clk = 1.8e9;
@@ -338,15 +416,20 @@ static void choose_config(const stencil_program *p, Launch &L) {
                     model(p, C);
                     int mrp = max_region_points(C);
                     for (int nt : cn) {
-                        if (!p->opt.threads && nt > rup(mrp, 32) && nt != cn.front()) continue;
+                        if (!p->opt.threads && (nt > tx * ty || nt > rup(mrp, 32)) && nt != cn.front())
+                            continue;
                         C.nt = nt;
+                        C.nth = nt + (p->opt.loader == 0 ? 32 : 0);
+                        C.est_regs = estimate_regs(p, C);
+                        if (C.est_regs > 255 && !(p->opt.threads && p->opt.tile_x)) continue;
+                        const int regs_alloc = (int)rup(std::min(C.est_regs, 255), 8);
                         C.ntx = (int)((g.nx + tx - 1) / tx);
                         C.nty = (int)((g.ny + ty - 1) / ty);
                         C.nch = (int)((nz + C.zc - 1) / C.zc);
                         double ctas = (double)C.ntx * C.nty * C.nch;
                         int per_sm = (int)std::min<int64_t>(
-                            {(int64_t)(228 * 1024 / (C.smem + 1024)), (int64_t)(2048 / nt), 32,
-                             (int64_t)(65536 / (nt * 64))});
+                            {(int64_t)(228 * 1024 / (C.smem + 1024)), (int64_t)(2048 / C.nth), 32,
+                             (int64_t)(65536 / (C.nth * regs_alloc))});
                         if (per_sm < 1) continue;
                         double slots = sms * per_sm;
                         double waves = std::ceil(ctas / slots);
@@ -355,6 +438,8 @@ static void choose_config(const stencil_program *p, Launch &L) {
                         double t_mem = C.bytes_exec * pts / hbm;
                         double t_sm = C.smem_pt * pts / smem_bw;
                         double t_alu = C.flops_exec * pts / alu;
+                        // issue rate: 4 warp-instructions per SM per cycle at ~60 % efficiency
+                        double t_issue = estimate_instr(C) * pts / 32.0 / (sms * 4 * clk * 0.6);
                         // idle lanes: points per thread rounding
                         double lanes = 0, used = 0;
                         for (const Stage &G : C.st) {
@@ -364,7 +449,7 @@ static void choose_config(const stencil_program *p, Launch &L) {
                             lanes += std::ceil(rp / nt) * nt;
                         }
                         t_alu *= lanes / std::max(used, 1.0);
-                        double t = std::max({t_mem, t_sm, t_alu}) / fill;
+                        double t = std::max({t_mem, t_sm, t_alu, t_issue}) / fill;
                         // bytes in flight per SM (latency hiding): want >= 32 KB
                         double inflight = 0;
                         for (size_t i = 0; i < C.in.size(); ++i)
@@ -375,6 +460,7 @@ static void choose_config(const stencil_program *p, Launch &L) {
                         double warps = std::min<double>(per_sm, std::ceil(ctas / sms)) * nt / 32;
                         if (warps < 8) t *= 8.0 / warps;
                         t += 2e-6 * waves;  // launch + wave tail overheads
+                        C.t_model = t;
                         if (t < best_t) { best_t = t; best = C; }
                     }
                 }
@@ -540,6 +626,74 @@ void sf_plan_set_impl(stencil_program *p, int32_t n_groups, const int32_t *group
     p->plan_groups = groups;
     p->has_plan = true;
 }
+
+// ------------------------------------------------------------ greedy planner
+// Host-side plan search (NEXT #1 in SURVEY.md §8(f); the paper's GGA search,
+// P:L140 §3.2.4 and P:L274-276 §5.4, evaluates candidate fusions with a
+// performance model, penalising infeasible ones).  Units are fission pieces
+// (§4.1: a kernel starts fully fissioned); adjacent groups in program
+// order are merged greedily while the modelled step time drops.  A candidate
+// group that violates a hazard (R11) or fits no tile is infeasible.
+namespace sf {
+std::vector<std::vector<int>> greedy_plan(stencil_program *p) {
+    // units: fission pieces in program order
+    std::vector<std::vector<int>> groups;
+    for (size_t k = 0; k < p->kernels.size(); ++k) {
+        int nc = 0;
+        std::vector<int> comp = fission_components(p, (int)k, &nc);
+        std::vector<std::vector<int>> pieces(nc);
+        for (size_t i = 0; i < comp.size(); ++i) pieces[comp[i]].push_back(p->kernels[k].stmts[i]);
+        for (auto &pc : pieces) groups.push_back(pc);
+    }
+    std::map<std::pair<std::vector<int>, std::vector<int>>, double> cache;
+    const double launch_cost = 3e-6;
+    auto group_cost = [&](const std::vector<int> &mem, const std::set<int> &stored) {
+        std::vector<int> st(stored.begin(), stored.end());
+        auto key = std::make_pair(mem, st);
+        auto it = cache.find(key);
+        if (it != cache.end()) return it->second;
+        double c;
+        try {
+            Launch L = analyze_group(p, mem, stored);
+            if (L.dead) c = 0;
+            else {
+                choose_config(p, L, true);
+                c = L.t_model + launch_cost;
+            }
+        } catch (const Error &) {
+            c = 1e30;
+        }
+        cache[key] = c;
+        return c;
+    };
+    auto plan_cost = [&](const std::vector<std::vector<int>> &gs) {
+        std::vector<std::set<int>> stored;
+        live_out(p, true, gs, stored);
+        double t = 0;
+        for (size_t g = 0; g < gs.size(); ++g) t += group_cost(gs[g], stored[g]);
+        return t;
+    };
+    double cur = plan_cost(groups);
+    for (;;) {
+        double best = cur;
+        size_t best_i = 0;
+        for (size_t i = 0; i + 1 < groups.size(); ++i) {
+            std::vector<std::vector<int>> cand = groups;
+            cand[i].insert(cand[i].end(), cand[i + 1].begin(), cand[i + 1].end());
+            std::sort(cand[i].begin(), cand[i].end());
+            cand.erase(cand.begin() + i + 1);
+            double c = plan_cost(cand);
+            if (c < best - 1e-9) { best = c; best_i = i; }
+        }
+        if (best >= cur) break;
+        groups[best_i].insert(groups[best_i].end(), groups[best_i + 1].begin(), groups[best_i + 1].end());
+        std::sort(groups[best_i].begin(), groups[best_i].end());
+        groups.erase(groups.begin() + best_i + 1);
+        cur = best;
+    }
+    return groups;
+}
+}  // namespace sf
 
 void sf_unfused_prepare(stencil_program *p) {
     if (p->unfused.analyzed) return;

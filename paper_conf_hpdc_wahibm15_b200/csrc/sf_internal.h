@@ -79,16 +79,20 @@ struct Launch {
     int z_below = 0, z_above = 0;
     // configuration
     int tx = 0, ty = 0, zc = 0, nt = 0, pf = 0;
+    int nth = 0;                 // threads per CTA (compute threads nt + producer warp)
+    int est_regs = 0;            // register estimate used by the tile chooser
+    double t_model = 0;          // modelled launch time (s)
     int ntx = 0, nty = 0, nch = 0;
     int64_t smem = 0;
     int rw_pad = 2;              // input row padding granularity (elements)
     // layout of smem (bytes) per input ring / stage ring
     std::vector<int64_t> in_off, in_plane;   // plane size in elements (padded)
-    std::vector<int> in_rw, in_rh;
+    std::vector<int> in_rw, in_rh, in_depth;  // ring depth: power of two
     std::vector<int64_t> st_off, st_plane;
-    std::vector<int> st_w, st_h;
+    std::vector<int> st_w, st_h, st_depth;
     int64_t bar_off = 0;
     int n_bars = 0;
+    int nbar_full = 1, nbar_empty = 1;  // per-step batch barriers (powers of two)
     // report
     double bytes_alg = 0, flops_alg = 0, bytes_exec = 0, flops_exec = 0, smem_pt = 0;
     // jit
@@ -155,9 +159,11 @@ std::vector<int> fission_components(const stencil_program *p, int kernel, int *n
 void analyze_mode(stencil_program *p, bool fused, const std::vector<std::vector<int>> &groups,
                   Mode &out);
 void fill_report(const stencil_program *p, const Launch &L, sp_group_report *r);
+std::vector<std::vector<int>> greedy_plan(stencil_program *p);
 
 // codegen.cpp
 std::string generate_launch(const stencil_program *p, Launch &L, int index, bool fused);
+void core_geometry(const Launch &L, int *xt, int *yt, int *cpx, int *cpy);
 
 // jit.cpp
 void compile_mode(stencil_program *p, Mode &m);

@@ -106,3 +106,22 @@ def test_c1_fused_equals_unfused_bitexact_perf_build(cuda_device):
     a = gpu_run(prog, "unfused", 1)
     b = gpu_run(prog, "fused", 1, plan=prog["plans"]["fused"])
     assert a["B"].tobytes() == b["B"].tobytes()
+
+
+def _c4_small():
+    import json as _json
+    from synth.scale_les import c4
+    prog = c4(nx=96, ny=32, nz=21)
+    prog["plans"]["fused"] = _json.load(open(os.path.join(os.path.dirname(os.path.dirname(
+        os.path.abspath(__file__))), "configs", "c4_plan.json")))["groups"]
+    return prog
+
+
+@pytest.mark.parametrize("fmad", [0, 1])
+def test_c4_parity_reduced(cuda_device, fmad):
+    """SCALE-LES-shaped 40-kernel DAG (BASELINE configs[3]) on a reduced grid, frozen greedy plan."""
+    prog = _c4_small()
+    ref = oracle_outputs(prog, seed=7)
+    for mode in ("unfused", "fused"):
+        got = gpu_run(prog, mode, 7, options={"fmad": fmad}, plan=prog["plans"]["fused"])
+        assert_close(prog, got, ref, exact=(fmad == 0))

@@ -1,9 +1,5 @@
 export PYTHONUNBUFFERED=1
-timeout 900 python -m pytest tests/test_gpu_parity.py -q -x 2>&1 | tail -15 > gpurun_out/t7.log
-timeout 200 python tools/quick_time.py C2 > gpurun_out/qt7_c2.log 2>&1
-timeout 200 python tools/quick_time.py C3 > gpurun_out/qt7_c3.log 2>&1
-for o in "--opt tile_x=32 --opt tile_y=8 --opt zchunk=64 --opt threads=64" "--opt tile_x=32 --opt tile_y=8 --opt zchunk=64 --opt threads=128" "--opt tile_x=32 --opt tile_y=16 --opt zchunk=64 --opt threads=128" "--opt tile_x=64 --opt tile_y=8 --opt zchunk=32 --opt threads=128" "--opt tile_x=32 --opt tile_y=16 --opt zchunk=32 --opt threads=64" "--opt tile_x=32 --opt tile_y=32 --opt zchunk=32 --opt threads=128" "--opt tile_x=32 --opt tile_y=8 --opt zchunk=32 --opt threads=64 --opt prefetch=2"; do
-  echo "== $o" >> gpurun_out/qt7_sweep.log
-  timeout 100 python tools/quick_time.py C2 fused $o 2>&1 | grep -E "fused|unfused :" >> gpurun_out/qt7_sweep.log
-done
-tail -3 gpurun_out/t7.log
+timeout 600 ncu --metrics gpu__time_duration.sum --clock-control none -k regex:sf_ --csv --log-file gpurun_out/launches9.csv python tools/prof_step.py C4 --steps 2 --warmup 1 --unfused > /dev/null 2>&1
+timeout 600 ncu --set full --clock-control none --import-source on -k regex:sf_fused_0 -c 1 -o gpurun_out/prof_c4f0 python tools/prof_step.py C4 --steps 1 --warmup 0 > gpurun_out/ncu9.log 2>&1
+timeout 600 ncu --set full --clock-control none --import-source on -k regex:sf_fused_6 -c 1 -o gpurun_out/prof_c4f6 python tools/prof_step.py C4 --steps 1 --warmup 0 >> gpurun_out/ncu9.log 2>&1
+tail -2 gpurun_out/ncu9.log

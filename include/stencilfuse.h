@@ -127,6 +127,8 @@ typedef struct {
     double bytes_exec;        /* incl. halo re-reads and z warm-up planes         */
     double flops_exec;        /* incl. halo recompute and warm-up                 */
     double smem_bytes_pt;     /* shared-memory traffic per point (model)          */
+    int32_t block_x, block_y, block_cby; /* per-thread register block of the core  */
+    double t_model_us;        /* modelled launch time (tile chooser objective)    */
 } sp_group_report;
 
 typedef struct sp_comm_s sp_comm;
@@ -199,6 +201,12 @@ sp_status sp_plan_report(const stencil_program *prog, int32_t mode, int32_t laun
 sp_status fusion_plan_report(const stencil_program *prog, int32_t group, sp_group_report *out);
 /* Generated CUDA source of a mode (for inspection); *len receives the full size. */
 sp_status sp_plan_source(stencil_program *prog, int32_t mode, char *buf, size_t cap, size_t *len);
+/* Halo-exchange schedule of one launch on several ranks: the arrays it reads
+ * beyond the local slab (up to cap written to arrays[], *n = total) and the
+ * exchange depth (its accumulated z reach, <= zhalo).  run_fused performs
+ * exactly this exchange before the launch's boundary chunks. */
+sp_status sp_plan_exchange(stencil_program *prog, int32_t mode, int32_t launch, int32_t cap,
+                           int32_t *arrays, int32_t *n, int32_t *depth);
 /* JIT-compile (NVRTC, sm_100a) without launching; needs no GPU. */
 sp_status sp_compile(stencil_program *prog, int32_t mode);
 

@@ -252,6 +252,14 @@ class Program:
         _check(lib().sp_plan_source(self.handle, self._mode(mode), buf, n.value + 1, ctypes.byref(n)))
         return buf.value.decode()
 
+    def exchange_plan(self, mode, i):
+        """(array names, depth) the executor exchanges before launch i on several ranks."""
+        n, depth = ctypes.c_int32(), ctypes.c_int32()
+        buf = (ctypes.c_int32 * len(self.names))()
+        _check(lib().sp_plan_exchange(self.handle, self._mode(mode), i, len(self.names), buf,
+                                      ctypes.byref(n), ctypes.byref(depth)))
+        return [self.names[buf[j]] for j in range(n.value)], depth.value
+
     def compile(self, mode):
         _check(lib().sp_compile(self.handle, self._mode(mode)))
 

@@ -66,7 +66,9 @@ class SpGroupReport(ctypes.Structure):
                 ("grid_ctas", ctypes.c_int32), ("regs_per_thread", ctypes.c_int32),
                 ("smem_bytes", ctypes.c_int64), ("bytes_alg", ctypes.c_double),
                 ("flops_alg", ctypes.c_double), ("bytes_exec", ctypes.c_double),
-                ("flops_exec", ctypes.c_double), ("smem_bytes_pt", ctypes.c_double)]
+                ("flops_exec", ctypes.c_double), ("smem_bytes_pt", ctypes.c_double),
+                ("block_x", ctypes.c_int32), ("block_y", ctypes.c_int32),
+                ("block_cby", ctypes.c_int32), ("t_model_us", ctypes.c_double)]
 
 
 # every symbol include/stencilfuse.h declares (checked by tests/test_abi.py)
@@ -75,7 +77,7 @@ EXPORTS = [
     "stencil_program_destroy", "stencil_program_layout", "stencil_program_bind",
     "sp_program_set_option", "sp_program_counts", "sp_program_edges", "sp_fission_components",
     "fusion_plan_set", "sp_plan_greedy", "sp_plan_count", "sp_plan_report", "fusion_plan_report", "sp_plan_source",
-    "sp_compile", "run_unfused", "run_fused", "sp_run_launch", "exchange_halos", "sp_last_error",
+    "sp_plan_exchange", "sp_compile", "run_unfused", "run_fused", "sp_run_launch", "exchange_halos", "sp_last_error",
 ]
 
 _lib = None
@@ -107,6 +109,7 @@ def lib():
             "fusion_plan_report": [vp, i32, P(SpGroupReport)],
             "sp_plan_source": [vp, i32, ctypes.c_char_p, ctypes.c_size_t, P(ctypes.c_size_t)],
             "sp_compile": [vp, i32],
+            "sp_plan_exchange": [vp, i32, i32, i32, P(i32), P(i32), P(i32)],
             "run_unfused": [vp, vp],
             "run_fused": [vp, vp],
             "sp_run_launch": [vp, i32, i32, vp],

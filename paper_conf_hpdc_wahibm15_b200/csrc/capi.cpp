@@ -77,6 +77,14 @@ static void interior_chunks(const stencil_program *p, const Launch &L, int *lo, 
     *hi = b;
 }
 
+// inputs a launch reads beyond the local slab, and the exchange depth (its z reach)
+static int exchange_set(const Launch &L, std::vector<int> &arrays) {
+    arrays.clear();
+    for (const Input &I : L.in)
+        if (I.qlo < 0 || I.ahi > 0) arrays.push_back(I.arr);
+    return std::max(L.z_below, L.z_above);
+}
+
 static void run_mode(stencil_program *p, int mode, void *stream) {
     Mode &m = mode_of(p, mode);
     load_mode(p, m);
@@ -84,10 +92,8 @@ static void run_mode(stencil_program *p, int mode, void *stream) {
     for (size_t i = 0; i < m.launches.size(); ++i) {
         Launch &L = m.launches[i];
         if (L.dead) continue;
-        int depth = std::max(L.z_below, L.z_above);
         std::vector<int> xarr;
-        for (const Input &I : L.in)
-            if (I.qlo < 0 || I.ahi > 0) xarr.push_back(I.arr);
+        int depth = exchange_set(L, xarr);
         if (!multi || depth == 0 || xarr.empty()) {
             launch(p, m, (int)i, stream, 0, 1, L.nch);
             continue;
@@ -192,6 +198,10 @@ sp_status sp_program_set_option(stencil_program *p, const char *key, int64_t v) 
         else if (k == "prefetch") o.prefetch = (int)v;
         else if (k == "num_sms") p->num_sms = (int)v;
         else if (k == "loader") o.loader = (int)v;
+        else if (k == "block_x") o.block_x = (int)v;
+        else if (k == "block_y") o.block_y = (int)v;
+        else if (k == "block_cby") o.block_cby = (int)v;
+        else if (k == "zqueue") o.zqueue = (int)v;
         else if (k == "l2_flush") {}
         else fail(SP_E_ARG, "unknown option '" + k + "'");
         if (v < 0 && k != "prefetch") fail(SP_E_ARG, "negative option value");
@@ -299,6 +309,19 @@ sp_status sp_plan_source(stencil_program *p, int32_t mode, char *buf, size_t cap
             std::memcpy(buf, all.data(), n);
             buf[n] = 0;
         }
+    });
+}
+
+sp_status sp_plan_exchange(stencil_program *p, int32_t mode, int32_t launch, int32_t cap,
+                           int32_t *arrays, int32_t *n, int32_t *depth) {
+    return guard([&] {
+        if (!p || !n || !depth) fail(SP_E_ARG, "null argument");
+        Mode &m = mode_of(p, mode);
+        if (launch < 0 || launch >= (int)m.launches.size()) fail(SP_E_ARG, "launch index out of range");
+        std::vector<int> a;
+        *depth = m.launches[launch].dead ? 0 : exchange_set(m.launches[launch], a);
+        *n = (int)a.size();
+        for (int i = 0; i < std::min<int>(cap, (int)a.size()); ++i) arrays[i] = a[i];
     });
 }
 

@@ -15,18 +15,21 @@
 //     §5.5.3), store live-out statements on the tile (reading R6) and arrive on
 //     the step's empty mbarrier.
 //
-// Thread mapping.  The tile core (TX x TY) is shared by all statements: thread t
-// owns the CP = (TX/XT) * ceil(TY/YT) points (xt + jx*XT, yt + iy*YT), so every
-// operand of a core point is a shared-memory load at a compile-time offset from
-// one per-step base register.  The halo strips of an extended region (the extra
-// layers of complex fusion) are enumerated per region class and spread over the
-// threads with small per-point tables.  Register-resident statements keep the
-// same mapping as their consumers (reading R7).
+// Register blocking of the tile core.  Thread (xt, yt) owns CBY blocks of VX x VY
+// points: block b covers x in [xt*VX, xt*VX+VX), y in [(b*YT+yt)*VY, +VY).  For a
+// statement, every shared-memory value its block needs (all taps of all VX*VY
+// points) is loaded once, 16-byte vectorised where aligned; a value needed at
+// several planes (z taps) is kept in a register queue that advances one plane
+// per step and is refilled by one load of the newest plane.  This divides the
+// shared-memory traffic per point — the binding resource of fused stencil
+// groups on B200 (SMEM : HBM bandwidth is only ~5.5 : 1) — by the reuse factor.
+// Halo strips (the extra layers of complex fusion) are evaluated point-wise.
 //
 // Ghost points (reading R1): a point outside the global interior takes the
-// array's ghost value through a predicated load.  CTAs whose tile lies inside the
-// interior run a core path without any per-point test.
+// array's ghost value through a predicated load; tiles inside the interior skip
+// the test.
 #include <cstdio>
+#include <functional>
 #include <set>
 #include <sstream>
 #include <tuple>
@@ -43,8 +46,7 @@ static std::string lit(double c, bool f32) {
 }
 
 static std::string num(int64_t v) { return std::to_string(v); }
-
-static std::string zname(int c) { return c < 0 ? "m" + num(-c) : "p" + num(c); }
+static std::string sg(int v) { return v < 0 ? "m" + num(-v) : "p" + num(v); }
 
 static int log2i(int v) {
     int l = 0;
@@ -52,40 +54,93 @@ static int log2i(int v) {
     return l;
 }
 
-namespace {
-// shared-memory layout a point indexes into: ring of input `a` or of stage `m`
-struct Lay {
-    bool stage;
-    int id;
-    bool operator<(const Lay &o) const { return std::tie(stage, id) < std::tie(o.stage, o.id); }
-};
-}  // namespace
-
-void core_geometry(const Launch &L, int *xt, int *yt, int *cpx, int *cpy) {
-    *xt = std::min(L.tx, L.nt);
+void core_geometry(const Launch &L, int *xt, int *yt) {
+    *xt = L.tx / L.vx;
     *yt = L.nt / *xt;
-    *cpx = L.tx / *xt;
-    *cpy = (L.ty + *yt - 1) / *yt;
 }
 
-// halo points of a region class: extended region minus the tile core
-static int halo_count(const Launch &L, const RegionClass &R) {
-    const int W = L.tx + R.x1 - R.x0, H = L.ty + R.y1 - R.y0;
-    return W * H - L.tx * L.ty;
+// ------------------------------------------------------------ position analysis
+// Values a statement's core block needs: (layout, y, x) relative to the block
+// origin, with the range of plane offsets c = lead + dz it is needed at.
+struct PosKey {
+    bool stage;
+    int id, y, x;
+    int c = 0;  // plane offset when z-queues are disabled (0 otherwise)
+    bool operator<(const PosKey &o) const {
+        return std::tie(stage, id, y, x, c) < std::tie(o.stage, o.id, o.y, o.x, o.c);
+    }
+};
+struct PosInfo { int cmin = 1 << 20, cmax = -(1 << 20); };
+
+static std::map<PosKey, PosInfo> block_positions(const Launch &L, const Stage &G) {
+    std::map<PosKey, PosInfo> pos;
+    for (const TermR &t : G.terms)
+        for (int w = 0; w < 2; ++w) {
+            if (w == 1 && !t.has_b) continue;
+            const Src &s = w ? t.b : t.a;
+            if (s.stage && L.st[s.idx].keep == Keep::Reg) continue;
+            for (int iy = 0; iy < L.vy; ++iy)
+                for (int jx = 0; jx < L.vx; ++jx) {
+                    int c = G.lead + s.dz;
+                    PosInfo &pi = pos[PosKey{s.stage, s.idx, iy + s.dy, jx + s.dx, L.zq ? 0 : c}];
+                    pi.cmin = std::min(pi.cmin, c);
+                    pi.cmax = std::max(pi.cmax, c);
+                }
+        }
+    return pos;
+}
+
+// registers the generated code keeps live (chooser's occupancy model)
+int codegen_regs(const stencil_program *p, const Launch &L) {
+    const int w = p->elem / 4;
+    int persistent = 0, transient = 0;
+    for (const Stage &G : L.st) {
+        if (!G.needed) continue;
+        auto pos = block_positions(L, G);
+        int direct = 0;
+        for (auto &kv : pos) {
+            int d = kv.second.cmax - kv.second.cmin + 1;
+            if (d > 1) persistent += d * L.cby * w;
+            else direct++;
+        }
+        transient = std::max(transient, (direct + L.vx * L.vy) * w);
+        if (G.keep == Keep::Reg) persistent += L.vx * L.vy * L.cby * G.depth * w;
+    }
+    int halo = 0;
+    for (const RegionClass &R : L.cls) {
+        int nh = (L.tx + R.x1 - R.x0) * (L.ty + R.y1 - R.y0) - L.tx * L.ty;
+        halo += (nh + L.nt - 1) / L.nt * 6;
+    }
+    return 48 + persistent + transient + halo + 2 * (int)L.in.size();
+}
+
+// shared-memory loads per core point over all statements (z-queue refills count
+// once per step; direct loads once per block position)
+double codegen_smem_loads(const Launch &L) {
+    double loads = 0;
+    for (const Stage &G : L.st) {
+        if (!G.needed) continue;
+        loads += (double)block_positions(L, G).size() / (L.vx * L.vy);
+    }
+    return loads;
 }
 
 std::string generate_launch(const stencil_program *p, Launch &L, int index, bool fused) {
     const bool f32 = p->elem == 4;
     const char *T = f32 ? "float" : "double";
+    const char *T2 = f32 ? "float4" : "double2";  // 16-byte vector
+    const int VW = 16 / p->elem;                   // elements per vector
     const sp_grid &g = p->grid;
     const sp_layout &lay = p->layout;
     const bool tma = p->opt.loader == 0;
     std::ostringstream o;
     L.fn = std::string(fused ? "sf_fused_" : "sf_unfused_") + num(index);
     L.nth = L.nt + (tma ? 32 : 0);
-    int XT, YT, CPX, CPY;
-    core_geometry(L, &XT, &YT, &CPX, &CPY);
-    const int CP = CPX * CPY;
+    int XT, YT;
+    core_geometry(L, &XT, &YT);
+    const int VX = L.vx, VY = L.vy, CBY = L.cby, NPB = VX * VY;
+    if (YT * VY * CBY != L.ty || XT * VX != L.tx || XT * YT != L.nt)
+        fail(SP_E_RESOURCES, "internal: inconsistent block geometry");
     for (const RegionClass &R : L.cls)
         if (R.x0 > 0 || R.x1 < 0 || R.y0 > 0 || R.y1 < 0)
             fail(SP_E_RESOURCES, "internal: region class does not contain the tile");
@@ -113,11 +168,11 @@ std::string generate_launch(const stencil_program *p, Launch &L, int index, bool
     o << "// generated by stencilfuse codegen: " << (fused ? "fused group " : "original kernel ")
       << L.name << "\n#include \"sf_device.cuh\"\n";
     o << "namespace " << L.fn << "_ns {\n";
-    o << "typedef " << T << " T;\n";
+    o << "typedef " << T << " T;\ntypedef " << T2 << " T2;\n";
     o << "constexpr int TX = " << L.tx << ", TY = " << L.ty << ", NT = " << L.nt << ", ZC = " << L.zc
       << ", KF = " << L.kfirst << ", PF = " << L.pf << ";\n";
-    o << "constexpr int XT = " << XT << ", YT = " << YT << ", CPX = " << CPX << ", CPY = " << CPY
-      << ";  // core: thread (xt, yt) owns (xt + jx*XT, yt + iy*YT)\n";
+    o << "constexpr int XT = " << XT << ", YT = " << YT << ", VX = " << VX << ", VY = " << VY
+      << ", CBY = " << CBY << ";  // thread (xt,yt) owns CBY blocks of VX x VY core points\n";
     o << "constexpr int NX = " << g.nx << ", NY = " << g.ny << ", NZ = " << g.nz_local
       << ", ZLO = " << p->zint_lo << ", ZHI = " << p->zint_hi << ";\n";
     o << "constexpr int XP = " << lay.x_pitch << ", YA = " << lay.y_alloc << ", ZA = " << lay.z_alloc
@@ -150,7 +205,7 @@ std::string generate_launch(const stencil_program *p, Launch &L, int index, bool
         if (G.keep == Keep::Smem)
             o << "  T *const st" << m << " = (T *)(sf_smem + " << L.st_off[m] << ");  // "
               << p->arrays[G.out].name << ": " << L.st_w[m] << "x" << L.st_h[m] << " x "
-              << L.st_depth[m] << " planes\n";
+              << L.st_depth[m] << " planes, cols " << -G.sx0 << "..\n";
     }
 
     // ------------------------------------------------------------ loads
@@ -219,33 +274,42 @@ std::string generate_launch(const stencil_program *p, Launch &L, int index, bool
         o << "      }\n    }\n    return;\n  }\n";
     }
 
-    // ---------------------------------------------------- layouts per class
-    std::vector<std::set<Lay>> lays(L.cls.size());
+    // ---------------------------------------------------- layouts
+    struct Lay {
+        bool stage;
+        int id;
+        bool operator<(const Lay &x) const { return std::tie(stage, id) < std::tie(x.stage, x.id); }
+    };
+    auto lw = [&](const Lay &l) { return l.stage ? L.st_w[l.id] : L.in_rw[l.id]; };
+    auto lx0 = [&](const Lay &l) { return l.stage ? -L.st[l.id].sx0 : -L.in[l.id].bx0; };
+    auto ly0 = [&](const Lay &l) { return l.stage ? -L.st[l.id].ey0 : -L.in[l.id].ey0; };
+    auto lname = [&](const Lay &l) { return std::string(l.stage ? "S" : "I") + num(l.id); };
+    std::vector<std::set<Lay>> hlays(L.cls.size());
     std::set<Lay> all_lays;
     for (size_t m = 0; m < L.st.size(); ++m) {
         const Stage &G = L.st[m];
         if (!G.needed) continue;
-        if (G.keep == Keep::Smem) lays[G.cls].insert(Lay{true, (int)m});
+        if (G.keep == Keep::Smem) {
+            hlays[G.cls].insert(Lay{true, (int)m});
+            all_lays.insert(Lay{true, (int)m});
+        }
         for (const TermR &t : G.terms)
             for (int w = 0; w < 2; ++w) {
                 if (w == 1 && !t.has_b) continue;
                 const Src &s = w ? t.b : t.a;
-                if (!s.stage) lays[G.cls].insert(Lay{false, s.idx});
-                else if (L.st[s.idx].keep == Keep::Smem) lays[G.cls].insert(Lay{true, s.idx});
+                if (s.stage && L.st[s.idx].keep == Keep::Reg) continue;
+                hlays[G.cls].insert(Lay{s.stage, s.idx});
+                all_lays.insert(Lay{s.stage, s.idx});
             }
     }
-    for (auto &st : lays) all_lays.insert(st.begin(), st.end());
-    auto lw = [&](const Lay &l) { return l.stage ? L.st_w[l.id] : L.in_rw[l.id]; };
-    auto lx0 = [&](const Lay &l) { return l.stage ? -L.st[l.id].ex0 : -L.in[l.id].bx0; };
-    auto ly0 = [&](const Lay &l) { return l.stage ? -L.st[l.id].ey0 : -L.in[l.id].ey0; };
-    auto lname = [&](const Lay &l) { return std::string(l.stage ? "S" : "I") + num(l.id); };
 
     // ---------------------------------------------------- per-thread core tables
     o << "  const int xt = tid % XT, yt = tid / XT;\n";
+    o << "  // core block b origin: (xt*VX, (b*YT + yt)*VY); index of its (0,0) in each layout\n";
     for (const Lay &l : all_lays)
-        o << "  const int cb_" << lname(l) << " = (yt - (" << ly0(l) << ")) * " << lw(l)
-          << " + (xt - (" << lx0(l) << "));\n";
-    o << "  const int cg = (Y0 + yt + OYA) * XP + X0 + xt + OXA;  // core point (0,0) in a plane\n";
+        o << "  const int cb_" << lname(l) << " = (yt * VY - (" << ly0(l) << ")) * " << lw(l)
+          << " + (xt * VX - (" << lx0(l) << "));\n";
+    o << "  const int cg = (Y0 + yt * VY + OYA) * XP + X0 + xt * VX + OXA;\n";
     o << "  const bool tile_in = X0 + TX <= NX && Y0 + TY <= NY;  // all core points interior\n";
 
     // halo tables per class
@@ -253,15 +317,14 @@ std::string generate_launch(const stencil_program *p, Launch &L, int index, bool
     for (size_t c = 0; c < L.cls.size(); ++c) {
         const RegionClass &R = L.cls[c];
         const int W = L.tx + R.x1 - R.x0, H = L.ty + R.y1 - R.y0;
-        nh[c] = halo_count(L, R);
+        nh[c] = W * H - L.tx * L.ty;
         hp[c] = (nh[c] + L.nt - 1) / L.nt;
         o << "  // class " << c << ": x [" << R.x0 << ", TX+" << R.x1 << "), y [" << R.y0 << ", TY+"
-          << R.y1 << "), " << W << "x" << H << ": core " << CP << " + halo " << nh[c] << " ("
-          << hp[c] << " per thread)\n";
+          << R.y1 << "), " << W << "x" << H << ": halo " << nh[c] << " points (" << hp[c]
+          << " per thread)\n";
         if (!nh[c]) continue;
         o << "  int h" << c << "_f[" << hp[c] << "], h" << c << "_g[" << hp[c] << "];\n";
-        for (const Lay &l : lays[c]) o << "  int h" << c << "_" << lname(l) << "[" << hp[c] << "];\n";
-        // enumerate halo points: rows above/below the tile at full width, then side columns
+        for (const Lay &l : hlays[c]) o << "  int h" << c << "_" << lname(l) << "[" << hp[c] << "];\n";
         const int top = -R.y0, bot = R.y1, left = -R.x0, right = R.x1;
         o << "  #pragma unroll\n  for (int i = 0; i < " << hp[c] << "; ++i) {\n";
         o << "    int e = min(tid + i * NT, " << nh[c] - 1 << "), x, y;\n";
@@ -276,18 +339,31 @@ std::string generate_launch(const stencil_program *p, Launch &L, int index, bool
         o << "    h" << c << "_f[i] = ((gx >= 0 && gx < NX && gy >= 0 && gy < NY) ? 2 : 0)"
           << " | ((ax >= 0 && ax < XP && ay >= 0 && ay < YA) ? 8 : 0);\n";
         o << "    h" << c << "_g[i] = ay * XP + ax;\n";
-        for (const Lay &l : lays[c])
+        for (const Lay &l : hlays[c])
             o << "    h" << c << "_" << lname(l) << "[i] = (y - (" << ly0(l) << ")) * " << lw(l)
               << " + (x - (" << lx0(l) << "));\n";
         o << "  }\n";
     }
-    // register queues: core points then halo points of the class
+
+    // register stages (core blocks + halo points) and z-queues of block positions
+    std::vector<std::map<PosKey, PosInfo>> bpos(L.st.size());
     for (size_t m = 0; m < L.st.size(); ++m) {
         const Stage &G = L.st[m];
-        if (G.keep != Keep::Reg) continue;
-        o << "  T rq" << m << "[" << CP << "][" << G.depth << "];\n";
-        if (nh[G.cls]) o << "  T rh" << m << "[" << hp[G.cls] << "][" << G.depth << "];\n";
+        if (!G.needed) continue;
+        bpos[m] = block_positions(L, G);
+        if (G.keep == Keep::Reg) {
+            o << "  T rq" << m << "[CBY][" << NPB << "][" << G.depth << "];\n";
+            if (nh[G.cls]) o << "  T rh" << m << "[" << hp[G.cls] << "][" << G.depth << "];\n";
+        }
     }
+    auto qname = [&](int m, const PosKey &k) {
+        return "zq" + num(m) + "_" + (k.stage ? "S" : "I") + num(k.id) + "_" + sg(k.y) + "_" + sg(k.x);
+    };
+    for (size_t m = 0; m < L.st.size(); ++m)
+        for (auto &kv : bpos[m])
+            if (kv.second.cmax > kv.second.cmin)
+                o << "  T " << qname((int)m, kv.first) << "[CBY][" << kv.second.cmax - kv.second.cmin + 1
+                  << "];\n";
     if (!tma) {
         o << "  for (int j = KF; j < min(KF + PF, zc); ++j) {\n";
         batch(o, "    ");
@@ -314,12 +390,14 @@ std::string generate_launch(const stencil_program *p, Launch &L, int index, bool
             for (int w = 0; w < 2; ++w) {
                 if (w == 1 && !t.has_b) continue;
                 const Src &s = w ? t.b : t.a;
-                if (!s.stage) basekeys.insert({Lay{false, s.idx}, G.lead + s.dz});
-                else if (L.st[s.idx].keep == Keep::Smem)
-                    basekeys.insert({Lay{true, s.idx}, G.lead + s.dz});
+                if (s.stage && L.st[s.idx].keep == Keep::Reg) continue;
+                basekeys.insert({Lay{s.stage, s.idx}, G.lead + s.dz});
             }
+        for (auto &kv : bpos[m])  // queue fills at the first step read every plane offset
+            for (int c = kv.second.cmin; c <= kv.second.cmax; ++c)
+                basekeys.insert({Lay{kv.first.stage, kv.first.id}, c});
     }
-    auto bname = [&](const Lay &l, int c) { return "B" + lname(l) + "_" + zname(c); };
+    auto bname = [&](const Lay &l, int c) { return "B" + lname(l) + "_" + sg(c); };
     for (auto &bk : basekeys) {
         const Lay &l = bk.first;
         const int c = bk.second;
@@ -355,19 +433,54 @@ std::string generate_launch(const stencil_program *p, Launch &L, int index, bool
             dirty.clear();
         }
         const int c = G.cls;
+        const auto &pos = bpos[m];
         o << "    { // stmt " << p->kernels[S.kernel].name << ":" << S.local << " -> "
           << p->arrays[G.out].name << "  lead " << G.lead << ", planes [" << G.loff << ", zc-1+"
           << G.lead << "], ext (" << G.ex0 << "," << G.ex1 << "," << G.ey0 << "," << G.ey1 << ")"
           << (G.stored ? ", stored" : "") << (G.keep == Keep::Reg ? ", register" : ", smem ring")
           << " depth " << G.depth << "\n";
+        // register-stage queues advance every step
         if (G.keep == Keep::Reg && G.depth > 1) {
-            o << "      #pragma unroll\n      for (int i = 0; i < " << CP << "; ++i)\n"
-              << "        #pragma unroll\n        for (int d = 0; d < " << G.depth - 1 << "; ++d) rq"
-              << m << "[i][d] = rq" << m << "[i][d + 1];\n";
+            o << "      #pragma unroll\n      for (int b = 0; b < CBY; ++b)\n"
+              << "      #pragma unroll\n      for (int i = 0; i < " << NPB << "; ++i)\n"
+              << "      #pragma unroll\n      for (int d = 0; d < " << G.depth - 1 << "; ++d) rq" << m
+              << "[b][i][d] = rq" << m << "[b][i][d + 1];\n";
             if (nh[c])
                 o << "      #pragma unroll\n      for (int i = 0; i < " << hp[c] << "; ++i)\n"
-                  << "        #pragma unroll\n        for (int d = 0; d < " << G.depth - 1
-                  << "; ++d) rh" << m << "[i][d] = rh" << m << "[i][d + 1];\n";
+                  << "      #pragma unroll\n      for (int d = 0; d < " << G.depth - 1 << "; ++d) rh"
+                  << m << "[i][d] = rh" << m << "[i][d + 1];\n";
+        }
+        // address of a block position in a layout at plane offset cc
+        auto baddr = [&](const PosKey &k, int cc) {
+            Lay l{k.stage, k.id};
+            return bname(l, cc) + " + cb_" + lname(l) + " + b * (YT * VY * " + num(lw(l)) + ") + (" +
+                   num(k.y * lw(l) + k.x) + ")";
+        };
+        // z-queues: advance, refill the newest plane (every step: the pipeline is uniform)
+        bool any_q = false;
+        for (auto &kv : pos)
+            if (kv.second.cmax > kv.second.cmin) any_q = true;
+        if (any_q) {
+            o << "      #pragma unroll\n      for (int b = 0; b < CBY; ++b) {\n";
+            o << "        if (k == KF) {\n";
+            for (auto &kv : pos) {
+                const PosInfo &pi = kv.second;
+                if (pi.cmax == pi.cmin) continue;
+                for (int cc = pi.cmin; cc <= pi.cmax; ++cc)
+                    o << "          " << qname(m, kv.first) << "[b][" << cc - pi.cmin << "] = *("
+                      << baddr(kv.first, cc) << ");\n";
+            }
+            o << "        } else {\n";
+            for (auto &kv : pos) {
+                const PosInfo &pi = kv.second;
+                if (pi.cmax == pi.cmin) continue;
+                const std::string q = qname(m, kv.first);
+                for (int d = 0; d < pi.cmax - pi.cmin; ++d)
+                    o << "          " << q << "[b][" << d << "] = " << q << "[b][" << d + 1 << "];\n";
+                o << "          " << q << "[b][" << pi.cmax - pi.cmin << "] = *("
+                  << baddr(kv.first, pi.cmax) << ");\n";
+            }
+            o << "        }\n      }\n";
         }
         o << "      const int q = k + (" << G.lead << ");\n";
         o << "      if (q >= (" << G.loff << ") && q <= zc - 1 + (" << G.lead << ")) {\n";
@@ -375,92 +488,171 @@ std::string generate_launch(const stencil_program *p, Launch &L, int index, bool
         o << "        const bool zin = gz >= ZLO && gz < ZHI;\n";
         o << "        const bool zal = gz + OZA >= 0 && gz + OZA < ZA;\n";
         o << "        T *const gpl = p.arr[" << L.arr_slot[G.out] << "] + (long long)(gz + OZA) * PLANE;\n";
+        if (G.stored) o << "        const bool zst = q >= 0 && q < zc;\n";
+        o << "        const bool fast = tile_in && zin;\n";
 
-        // expression over operand accessors; mode 0 = core (iy, jx), 1 = halo (i)
-        auto operand = [&](const Src &s, int mode) -> std::string {
+        // ---- core blocks
+        o << "        #pragma unroll\n        for (int b = 0; b < CBY; ++b) {\n";
+        // direct loads, vectorised along x where aligned
+        std::map<std::tuple<bool, int, int, int>, std::set<int>> rows;  // (stage,id,c,y) -> xs
+        for (auto &kv : pos)
+            if (kv.second.cmax == kv.second.cmin)
+                rows[std::make_tuple(kv.first.stage, kv.first.id, kv.second.cmin, kv.first.y)].insert(
+                    kv.first.x);
+        auto dname = [&](bool st, int id, int cc, int y, int x) {
+            return std::string("d_") + (st ? "S" : "I") + num(id) + "_" + sg(cc) + "_" + sg(y) + "_" +
+                   sg(x);
+        };
+        const bool vec_ok = VW > 1 && VX % VW == 0;
+        for (auto &rw : rows) {
+            bool st;
+            int id, cc, y;
+            std::tie(st, id, cc, y) = rw.first;
+            const std::set<int> &xs = rw.second;
+            std::set<int> done;
+            for (int x : xs) {
+                if (done.count(x)) continue;
+                // 16-byte vector starting at an aligned x (block origins and layouts are aligned)
+                int xa = x - (((x % VW) + VW) % VW);
+                int cnt = 0;
+                for (int e2 = 0; e2 < VW; ++e2) cnt += (int)xs.count(xa + e2);
+                if (vec_ok && cnt >= 2) {
+                    std::string vn = "v" + dname(st, id, cc, y, xa);
+                    o << "          const T2 " << vn << " = *reinterpret_cast<const T2 *>("
+                      << baddr(PosKey{st, id, y, xa, 0}, cc) << ");\n";
+                    const char *comp[4] = {"x", "y", "z", "w"};
+                    for (int e2 = 0; e2 < VW; ++e2)
+                        if (xs.count(xa + e2)) {
+                            o << "          const T " << dname(st, id, cc, y, xa + e2) << " = " << vn
+                              << "." << comp[e2] << ";\n";
+                            done.insert(xa + e2);
+                        }
+                } else {
+                    o << "          const T " << dname(st, id, cc, y, x) << " = *("
+                      << baddr(PosKey{st, id, y, x, 0}, cc) << ");\n";
+                    done.insert(x);
+                }
+            }
+        }
+        // expressions of the VX*VY block points
+        auto core_operand = [&](const Src &s, int iy, int jx) -> std::string {
             if (s.stage && L.st[s.idx].keep == Keep::Reg) {
                 const Stage &P = L.st[s.idx];
                 int d = G.lead + s.dz - P.lead + P.depth - 1;
-                return std::string(mode == 0 ? "rq" : "rh") + num(s.idx) + "[" +
-                       (mode == 0 ? "iy * CPX + jx" : "i") + "][" + num(d) + "]";
+                return "rq" + num(s.idx) + "[b][" + num(iy * VX + jx) + "][" + num(d) + "]";
             }
-            Lay l{s.stage, s.idx};
             int cc = G.lead + s.dz;
-            int off = s.dy * lw(l) + s.dx;
-            if (mode == 0)
-                return bname(l, cc) + "[cb_" + lname(l) + " + iy * (YT * " + num(lw(l)) +
-                       ") + jx * XT + (" + num(off) + ")]";
-            return bname(l, cc) + "[h" + num(c) + "_" + lname(l) + "[i] + (" + num(off) + ")]";
+            PosKey k{s.stage, s.idx, iy + s.dy, jx + s.dx, L.zq ? 0 : cc};
+            const PosInfo &pi = pos.at(k);
+            if (pi.cmax > pi.cmin) return qname(m, k) + "[b][" + num(cc - pi.cmin) + "]";
+            return dname(s.stage, s.idx, cc, k.y, k.x);
         };
-        auto expr = [&](int mode) {
+        auto term_expr = [&](const std::function<std::string(const Src &)> &opd) {
             std::string e;
             for (size_t ti = 0; ti < G.terms.size(); ++ti) {
                 const TermR &t = G.terms[ti];
-                std::string a = operand(t.a, mode);
+                std::string a = opd(t.a);
                 std::string term;
                 if (t.coef == 1.0) term = a;
                 else if (t.coef == -1.0) term = "(-" + a + ")";
                 else term = "(T)" + lit(t.coef, f32) + " * " + a;
-                if (t.has_b) term = "(" + term + ") * " + operand(t.b, mode);
+                if (t.has_b) term = "(" + term + ") * " + opd(t.b);
                 e = ti == 0 ? term : "(" + e + ") + " + term;
             }
             return e;
         };
-        Lay self{true, m};
-        auto sink = [&](int mode, const std::string &pt_g, bool store_ok) {
-            std::ostringstream s;
-            if (G.keep == Keep::Smem) {
-                if (mode == 0)
-                    s << "            " << bname(self, G.lead) << "[cb_" << lname(self)
-                      << " + iy * (YT * " << lw(self) << ") + jx * XT] = v;\n";
-                else
-                    s << "            " << bname(self, G.lead) << "[h" << c << "_" << lname(self)
-                      << "[i]] = v;\n";
-            } else {
-                s << "            " << (mode == 0 ? "rq" : "rh") << m << "["
-                  << (mode == 0 ? "iy * CPX + jx" : "i") << "][" << G.depth - 1 << "] = v;\n";
+        for (int iy = 0; iy < VY; ++iy)
+            for (int jx = 0; jx < VX; ++jx)
+                o << "          T o" << iy << "_" << jx << " = "
+                  << term_expr([&](const Src &s) { return core_operand(s, iy, jx); }) << ";\n";
+        // ghost substitution and store predicates outside the interior (edge tiles, z ghosts)
+        o << "          const int by = (b * YT + yt) * VY;\n";
+        o << "          if (!fast) {\n";
+        for (int iy = 0; iy < VY; ++iy)
+            for (int jx = 0; jx < VX; ++jx) {
+                std::string gx = "X0 + xt * VX + " + num(jx), gy = "Y0 + by + " + num(iy);
+                o << "            if (!(zin && " << gx << " < NX && " << gy << " < NY)) o" << iy << "_"
+                  << jx << " = sf_ldg_pred(gpl + cg + b * (YT * VY * XP) + (" << iy << " * XP + " << jx
+                  << "), zal && " << gx << " < XP - OXA && " << gy << " < YA - OYA);\n";
             }
-            if (G.stored && mode == 0 && store_ok) s << "            sf_st(gpl + " << pt_g << ", v);\n";
-            return s.str();
-        };
-        const std::string core_g = "cg + iy * (YT * XP) + jx * XT";
-        // core, fast path: tile inside the interior, plane interior
-        if (G.stored) o << "        const bool zst = q >= 0 && q < zc;\n";
-        o << "        if (tile_in && zin) {\n";
-        o << "          #pragma unroll\n          for (int iy = 0; iy < CPY; ++iy)\n"
-          << "          #pragma unroll\n          for (int jx = 0; jx < CPX; ++jx) {\n";
-        if (L.ty % YT) o << "            if (yt + iy * YT >= TY) continue;\n";
-        o << "            T v = " << expr(0) << ";\n";
-        if (G.stored) {
-            std::string sk = sink(0, core_g, true);
-            // stores only for the chunk's own planes
-            auto pos = sk.find("            sf_st(");
-            if (pos != std::string::npos) sk.insert(pos + 12, "if (zst) ");
-            o << sk;
+        o << "          }\n";
+        // sinks
+        if (G.keep == Keep::Smem) {
+            Lay self{true, m};
+            for (int iy = 0; iy < VY; ++iy) {
+                std::string a = bname(self, G.lead) + " + cb_" + lname(self) + " + b * (YT * VY * " +
+                                num(lw(self)) + ") + (" + num(iy * lw(self)) + ")";
+                if (vec_ok) {
+                    for (int jx = 0; jx < VX; jx += VW) {
+                        o << "          *reinterpret_cast<T2 *>(" << a << " + " << jx << ") = T2{";
+                        for (int e2 = 0; e2 < VW; ++e2)
+                            o << (e2 ? ", " : "") << "o" << iy << "_" << jx + e2;
+                        o << "};\n";
+                    }
+                } else {
+                    for (int jx = 0; jx < VX; ++jx)
+                        o << "          *(" << a << " + " << jx << ") = o" << iy << "_" << jx << ";\n";
+                }
+            }
         } else {
-            o << sink(0, core_g, false);
+            for (int iy = 0; iy < VY; ++iy)
+                for (int jx = 0; jx < VX; ++jx)
+                    o << "          rq" << m << "[b][" << iy * VX + jx << "][" << G.depth - 1 << "] = o"
+                      << iy << "_" << jx << ";\n";
         }
-        o << "          }\n        } else {\n";
-        o << "          #pragma unroll\n          for (int iy = 0; iy < CPY; ++iy)\n"
-          << "          #pragma unroll\n          for (int jx = 0; jx < CPX; ++jx) {\n";
-        if (L.ty % YT) o << "            if (yt + iy * YT >= TY) continue;\n";
-        o << "            const bool in = zin && X0 + xt + jx * XT < NX && Y0 + yt + iy * YT < NY;\n";
-        o << "            T v = " << expr(0) << ";\n";
-        o << "            if (!in) v = sf_ldg_pred(gpl + (" << core_g << "), zal && X0 + xt + jx * XT < XP - OXA && Y0 + yt + iy * YT < YA - OYA);\n";
-        {
-            std::string sk = sink(0, core_g, G.stored);
-            auto pos = sk.find("            sf_st(");
-            if (pos != std::string::npos) sk.insert(pos + 12, "if (zst && in) ");
-            o << sk;
+        if (G.stored) {
+            o << "          if (zst) {\n";
+            o << "            T *const gb = gpl + cg + b * (YT * VY * XP);\n";
+            o << "            if (fast) {\n";
+            for (int iy = 0; iy < VY; ++iy) {
+                if (vec_ok) {
+                    for (int jx = 0; jx < VX; jx += VW) {
+                        o << "              sf_st_v(gb + (" << iy << " * XP + " << jx << "), T2{";
+                        for (int e2 = 0; e2 < VW; ++e2)
+                            o << (e2 ? ", " : "") << "o" << iy << "_" << jx + e2;
+                        o << "});\n";
+                    }
+                } else {
+                    for (int jx = 0; jx < VX; ++jx)
+                        o << "              sf_st(gb + (" << iy << " * XP + " << jx << "), o" << iy
+                          << "_" << jx << ");\n";
+                }
+            }
+            o << "            } else {\n";
+            for (int iy = 0; iy < VY; ++iy)
+                for (int jx = 0; jx < VX; ++jx)
+                    o << "              if (X0 + xt * VX + " << jx << " < NX && Y0 + by + " << iy
+                      << " < NY) sf_st(gb + (" << iy << " * XP + " << jx << "), o" << iy << "_" << jx
+                      << ");\n";
+            o << "            }\n          }\n";
         }
-        o << "          }\n        }\n";
+        o << "        }\n";
+
+        // ---- halo points (point-wise)
         if (nh[c]) {
+            auto halo_operand = [&](const Src &s) -> std::string {
+                if (s.stage && L.st[s.idx].keep == Keep::Reg) {
+                    const Stage &P = L.st[s.idx];
+                    int d = G.lead + s.dz - P.lead + P.depth - 1;
+                    return "rh" + num(s.idx) + "[i][" + num(d) + "]";
+                }
+                Lay l{s.stage, s.idx};
+                int off = s.dy * lw(l) + s.dx;
+                return bname(l, G.lead + s.dz) + "[h" + num(c) + "_" + lname(l) + "[i] + (" +
+                       num(off) + ")]";
+            };
             o << "        #pragma unroll\n        for (int i = 0; i < " << hp[c] << "; ++i) {\n";
             o << "          const int f = h" << c << "_f[i];\n";
-            o << "          T v = " << expr(1) << ";\n";
+            o << "          T v = " << term_expr(halo_operand) << ";\n";
             o << "          if (!(zin && (f & 2))) v = sf_ldg_pred(gpl + h" << c
               << "_g[i], zal && (f & 8));\n";
-            o << sink(1, "", false);
+            if (G.keep == Keep::Smem) {
+                Lay self{true, m};
+                o << "          " << bname(self, G.lead) << "[h" << c << "_" << lname(self)
+                  << "[i]] = v;\n";
+            } else {
+                o << "          rh" << m << "[i][" << G.depth - 1 << "] = v;\n";
+            }
             o << "        }\n";
         }
         o << "      }\n    }\n";

@@ -81,6 +81,17 @@ __device__ __forceinline__ void sf_st(double *p, double v) {
 __device__ __forceinline__ void sf_st(float *p, float v) {
     asm volatile("st.global.L1::no_allocate.f32 [%0], %1;" ::"l"(p), "f"(v) : "memory");
 }
+// 16-byte live-out stores (x-adjacent points of a register block)
+__device__ __forceinline__ void sf_st_v(double *p, double2 v) {
+    asm volatile("st.global.L1::no_allocate.v2.f64 [%0], {%1, %2};" ::"l"(p), "d"(v.x), "d"(v.y)
+                 : "memory");
+}
+__device__ __forceinline__ void sf_st_v(float *p, float4 v) {
+    asm volatile("st.global.L1::no_allocate.v4.f32 [%0], {%1, %2, %3, %4};" ::"l"(p), "f"(v.x),
+                 "f"(v.y), "f"(v.z), "f"(v.w)
+                 : "memory");
+}
+
 // ghost value of a point outside the global interior: predicated non-coherent
 // load (ghost cells are never written), 0 when the point is outside the allocation
 __device__ __forceinline__ double sf_ldg_pred(const double *p, bool pred) {

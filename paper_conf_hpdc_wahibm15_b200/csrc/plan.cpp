@@ -243,8 +243,9 @@ static void layout_launch(const stencil_program *p, Launch &L) {
     L.nbar_full = pow2ceil(L.pf + 1);
     L.nbar_empty = pow2ceil(L.pf + 2);
     L.n_bars = L.nbar_full + L.nbar_empty;
-    for (const Stage &G : L.st) {
-        int w = L.tx + G.ex0 + G.ex1, h = L.ty + G.ey0 + G.ey1;
+    for (Stage &G : L.st) {
+        G.sx0 = (int)rup(G.ex0, L.rw_pad);
+        int w = (int)rup(G.sx0 + L.tx + G.ex1, L.rw_pad), h = L.ty + G.ey0 + G.ey1;
         L.st_w.push_back(w);
         L.st_h.push_back(h);
         if (G.keep == Keep::Smem) {
@@ -270,60 +271,24 @@ static void layout_launch(const stencil_program *p, Launch &L) {
 // register estimate of a configured launch (occupancy model of the tile chooser;
 // the paper tunes block size with the occupancy-calculator equations, §4.2)
 static int estimate_regs(const stencil_program *p, const Launch &L) {
-    const int w64 = p->elem / 4;
-    int xt, yt, cpx, cpy;
-    core_geometry(L, &xt, &yt, &cpx, &cpy);
-    const int cp = cpx * cpy;
-    std::vector<std::set<int>> lays(L.cls.size());
-    std::set<int> all;
-    std::set<std::pair<int, int>> bases;
-    for (size_t m = 0; m < L.st.size(); ++m) {
-        const Stage &G = L.st[m];
-        if (!G.needed) continue;
-        if (G.keep == Keep::Smem) { lays[G.cls].insert(1000 + (int)m); bases.insert({1000 + (int)m, G.lead}); }
-        for (const TermR &t : G.terms)
-            for (int w = 0; w < 2; ++w) {
-                if (w == 1 && !t.has_b) continue;
-                const Src &s = w ? t.b : t.a;
-                if (!s.stage) { lays[G.cls].insert(s.idx); bases.insert({s.idx, G.lead + s.dz}); }
-                else if (L.st[s.idx].keep == Keep::Smem) {
-                    lays[G.cls].insert(1000 + s.idx);
-                    bases.insert({1000 + s.idx, G.lead + s.dz});
-                }
-            }
-    }
-    for (auto &st : lays) all.insert(st.begin(), st.end());
-    int regs = 40 + (int)all.size() + (int)bases.size();
-    std::vector<int> hp(L.cls.size());
-    for (size_t c = 0; c < L.cls.size(); ++c) {
-        const RegionClass &R = L.cls[c];
-        int nh = (L.tx + R.x1 - R.x0) * (L.ty + R.y1 - R.y0) - L.tx * L.ty;
-        hp[c] = (nh + L.nt - 1) / L.nt;
-        regs += hp[c] * (2 + (int)lays[c].size());
-    }
-    for (const Stage &G : L.st)
-        if (G.keep == Keep::Reg) regs += (cp + hp[G.cls]) * G.depth * w64;
-    regs += 3 * cp * w64;
-    return regs;
+    return codegen_regs(p, L);
 }
 
 // issued instructions per output point (thread-level), for the issue-rate ceiling
 static double estimate_instr(const Launch &L) {
-    int xt, yt, cpx, cpy;
-    core_geometry(L, &xt, &yt, &cpx, &cpy);
     const double tile = (double)L.tx * L.ty;
-    double per_pt = 0, per_step = 60;
+    double per_pt = codegen_smem_loads(L) * 1.2, per_step = 60;
     for (const Stage &G : L.st) {
         if (!G.needed) continue;
         double pts = (double)(L.tx + G.ex0 + G.ex1) * (L.ty + G.ey0 + G.ey1);
         double halo = pts - tile;
         int ops = 0;
-        for (const TermR &t : G.terms) ops += 2 + (t.has_b ? 2 : 0);
-        per_pt += (ops + 2) * 1.0 + (G.stored ? 1 : 0) + halo / tile * (ops + 10);
-        per_step += 12 + 4.0 * G.terms.size() / 2;
+        for (const TermR &t : G.terms) ops += 1 + (t.has_b ? 1 : 0);
+        per_pt += ops + 1 + (G.stored ? 0.5 : 0) + halo / tile * (2 * ops + 10);
+        per_step += 12;
     }
-    // per-step work is shared by the cp points of a thread
-    return per_pt + per_step / (cpx * cpy) * ((double)L.nt * cpx * cpy / tile);
+    // per-step work is shared by the points of a thread
+    return per_pt + per_step * L.nt / tile;
 }
 
 // per-point byte/flop model of a configured launch
@@ -349,8 +314,10 @@ static void model(const stencil_program *p, Launch &L) {
                 const Src &s = w ? t.b : t.a;
                 if (!s.stage || L.st[s.idx].keep == Keep::Smem) ++smem_reads;
             }
-        sm += (smem_reads + (G.keep == Keep::Smem ? 1 : 0)) * e * pts / tile;
+        const double core = (double)L.tx * L.ty * (L.zc - 1 + G.lead - G.loff + 1);
+        sm += (smem_reads * (pts - core) + (G.keep == Keep::Smem ? pts : 0)) * e / tile;
     }
+    sm += codegen_smem_loads(L) * e;
     double by_exec = n_store * (double)e;
     for (size_t i = 0; i < L.in.size(); ++i) {
         const Input &I = L.in[i];
@@ -377,99 +344,104 @@ static void choose_config(const stencil_program *p, Launch &L, bool quick = fals
     const sp_grid &g = p->grid;
     const int e = p->elem;
     const int64_t nz = g.nz_local;
-    std::vector<int> cx, cy, cz, cn, cp;
-    if (p->opt.tile_x) cx = {p->opt.tile_x};
+    const Options &o = p->opt;
+    std::vector<int> cx, cz, cn, cp, cvx, cvy, ccb;
+    if (o.tile_x) cx = {o.tile_x};
     else if (quick) cx = e == 8 ? std::vector<int>{32, 64} : std::vector<int>{64, 128};
     else cx = e == 8 ? std::vector<int>{16, 32, 64} : std::vector<int>{32, 64, 128};
-    if (p->opt.tile_y) cy = {p->opt.tile_y};
-    else if (quick) cy = {8, 16, 32};
-    else cy = {1, 2, 4, 8, 16, 32};
-    if (p->opt.zchunk) cz = {p->opt.zchunk};
+    if (o.zchunk) cz = {o.zchunk};
     else if (quick) cz = {16, 32, 64};
     else cz = {4, 8, 16, 32, 64, 128, 256, 512};
-    if (p->opt.threads) cn = {p->opt.threads};
+    if (o.threads) cn = {o.threads};
     else cn = {64, 128, 256};
-    if (p->opt.prefetch >= 0) cp = {p->opt.prefetch};
+    if (o.prefetch >= 0) cp = {o.prefetch};
     else if (quick) cp = {1, 2};
     else cp = {1, 2, 3};
+    if (o.block_x) cvx = {o.block_x};
+    else cvx = e == 8 ? std::vector<int>{1, 2} : std::vector<int>{1, 2, 4};
+    if (o.block_y) cvy = {o.block_y};
+    else cvy = {1, 2, 4};
+    if (o.block_cby) ccb = {o.block_cby};
+    else ccb = {1, 2, 4};
     const double sms = p->num_sms;
     const double clk = 1.8e9;
     const double hbm = 6.0e12, smem_bw = sms * 128 * clk;
     const double alu = sms * (e == 8 ? 64 : 128) * clk;
+    const double pts = (double)g.nx * g.ny * nz;
     Launch best;
     double best_t = 1e300;
     for (int tx : cx) {
-        if (!p->opt.tile_x && tx >= 2 * g.nx && tx != cx.front()) continue;
-        for (int ty : cy) {
-            if (!p->opt.tile_y && ty >= 2 * g.ny && ty != cy.front()) continue;
-            for (int zc : cz) {
-                if (!p->opt.zchunk && zc >= 2 * nz && zc != cz.front()) continue;
-                for (int pf : cp) {
-                    Launch C = L;
-                    C.tx = tx; C.ty = ty; C.zc = (int)std::min<int64_t>(zc, nz); C.pf = pf;
-                    layout_launch(p, C);
-                    if (C.smem > 227 * 1024) continue;
-                    bool box_ok = true;  // TMA box extents are limited to 256
-                    for (size_t i = 0; i < C.in.size(); ++i)
-                        if (C.in_rw[i] > 256 || C.in_rh[i] > 256) box_ok = false;
-                    if (!box_ok) continue;
-                    model(p, C);
-                    int mrp = max_region_points(C);
-                    for (int nt : cn) {
-                        if (!p->opt.threads && (nt > tx * ty || nt > rup(mrp, 32)) && nt != cn.front())
+        if (!o.tile_x && tx >= 2 * g.nx && tx != cx.front()) continue;
+        for (int vx : cvx) {
+            if (tx % vx) continue;
+            const int xt = tx / vx;
+            for (int nt : cn) {
+                if (nt % xt || xt > nt) continue;
+                const int yt = nt / xt;
+                for (int vy : cvy)
+                    for (int cby : ccb) {
+                        const int ty = yt * vy * cby;
+                        if (o.tile_y && ty != o.tile_y) continue;
+                        if (!o.tile_y && (ty > 64 || (ty >= 2 * g.ny && (vy > 1 || cby > 1))))
                             continue;
-                        C.nt = nt;
-                        C.nth = nt + (p->opt.loader == 0 ? 32 : 0);
-                        C.est_regs = estimate_regs(p, C);
-                        if (C.est_regs > 255 && !(p->opt.threads && p->opt.tile_x)) continue;
-                        const int regs_alloc = (int)rup(std::min(C.est_regs, 255), 8);
-                        C.ntx = (int)((g.nx + tx - 1) / tx);
-                        C.nty = (int)((g.ny + ty - 1) / ty);
-                        C.nch = (int)((nz + C.zc - 1) / C.zc);
-                        double ctas = (double)C.ntx * C.nty * C.nch;
-                        int per_sm = (int)std::min<int64_t>(
-                            {(int64_t)(228 * 1024 / (C.smem + 1024)), (int64_t)(2048 / C.nth), 32,
-                             (int64_t)(65536 / (C.nth * regs_alloc))});
-                        if (per_sm < 1) continue;
-                        double slots = sms * per_sm;
-                        double waves = std::ceil(ctas / slots);
-                        double fill = ctas / (waves * slots);
-                        double pts = (double)g.nx * g.ny * nz;
-                        double t_mem = C.bytes_exec * pts / hbm;
-                        double t_sm = C.smem_pt * pts / smem_bw;
-                        double t_alu = C.flops_exec * pts / alu;
-                        // issue rate: 4 warp-instructions per SM per cycle at ~60 % efficiency
-                        double t_issue = estimate_instr(C) * pts / 32.0 / (sms * 4 * clk * 0.6);
-                        // idle lanes: points per thread rounding
-                        double lanes = 0, used = 0;
-                        for (const Stage &G : C.st) {
-                            if (!G.needed) continue;
-                            double rp = (double)(tx + G.ex0 + G.ex1) * (ty + G.ey0 + G.ey1);
-                            used += rp;
-                            lanes += std::ceil(rp / nt) * nt;
+                        for (int zc : cz) {
+                            if (!o.zchunk && zc >= 2 * nz && zc != cz.front()) continue;
+                            for (int pf : cp) {
+                                Launch C = L;
+                                C.tx = tx; C.ty = ty; C.zc = (int)std::min<int64_t>(zc, nz);
+                                C.pf = pf; C.nt = nt; C.vx = vx; C.vy = vy; C.cby = cby;
+                                C.zq = o.zqueue;
+                                C.nth = nt + (o.loader == 0 ? 32 : 0);
+                                layout_launch(p, C);
+                                if (C.smem > 227 * 1024) continue;
+                                bool box_ok = true;  // TMA box extents are limited to 256
+                                for (size_t i = 0; i < C.in.size(); ++i)
+                                    if (C.in_rw[i] > 256 || C.in_rh[i] > 256) box_ok = false;
+                                if (!box_ok) continue;
+                                C.est_regs = estimate_regs(p, C);
+                                const bool forced = o.tile_x && o.block_x && o.block_y && o.block_cby &&
+                                                    o.threads;
+                                if (C.est_regs > 255 && !forced) continue;
+                                model(p, C);
+                                const int regs_alloc = (int)rup(std::min(C.est_regs, 255), 8);
+                                C.ntx = (int)((g.nx + tx - 1) / tx);
+                                C.nty = (int)((g.ny + ty - 1) / ty);
+                                C.nch = (int)((nz + C.zc - 1) / C.zc);
+                                double ctas = (double)C.ntx * C.nty * C.nch;
+                                int per_sm = (int)std::min<int64_t>(
+                                    {(int64_t)(228 * 1024 / (C.smem + 1024)), (int64_t)(2048 / C.nth),
+                                     32, (int64_t)(65536 / (C.nth * regs_alloc))});
+                                if (per_sm < 1) continue;
+                                double slots = sms * per_sm;
+                                double waves = std::ceil(ctas / slots);
+                                double fill = ctas / (waves * slots);
+                                double t_mem = C.bytes_exec * pts / hbm;
+                                double t_sm = C.smem_pt * pts / smem_bw;
+                                double t_alu = C.flops_exec * pts / alu;
+                                // issue rate: 4 warp-instructions per SM per cycle at ~70 %
+                                double t_issue = estimate_instr(C) * pts / 32.0 / (sms * 4 * clk * 0.7);
+                                // latency hiding by the compute warps (barrier-separated stages)
+                                double warps = std::min<double>(per_sm, std::ceil(ctas / sms)) * nt / 32;
+                                double lat = std::min(1.0, warps / 16.0);
+                                double t = std::max({t_mem, t_sm / lat, t_alu / lat, t_issue / lat}) / fill;
+                                // bytes in flight per SM (TMA latency hiding): want >= 40 KB
+                                double inflight = 0;
+                                for (size_t i = 0; i < C.in.size(); ++i)
+                                    inflight += (double)C.in_rw[i] * C.in_rh[i] * e * pf;
+                                inflight *= std::min<double>(per_sm, std::ceil(ctas / sms));
+                                if (inflight < 40960) t *= std::sqrt(40960.0 / std::max(inflight, 1024.0));
+                                t += 2e-6 * waves;  // launch + wave tail overheads
+                                C.t_model = t;
+                                if (t < best_t) { best_t = t; best = C; }
+                            }
                         }
-                        t_alu *= lanes / std::max(used, 1.0);
-                        double t = std::max({t_mem, t_sm, t_alu, t_issue}) / fill;
-                        // bytes in flight per SM (latency hiding): want >= 32 KB
-                        double inflight = 0;
-                        for (size_t i = 0; i < C.in.size(); ++i)
-                            inflight += (double)C.in_plane[i] * e * pf;
-                        inflight *= std::min<double>(per_sm, std::ceil(ctas / sms));
-                        if (inflight < 32768) t *= 32768.0 / std::max(inflight, 1024.0);
-                        // warps per SM for the compute part
-                        double warps = std::min<double>(per_sm, std::ceil(ctas / sms)) * nt / 32;
-                        if (warps < 8) t *= 8.0 / warps;
-                        t += 2e-6 * waves;  // launch + wave tail overheads
-                        C.t_model = t;
-                        if (t < best_t) { best_t = t; best = C; }
                     }
-                }
             }
         }
     }
     if (best_t >= 1e299)
         fail(SP_E_RESOURCES, "group '" + L.name + "': no tile configuration fits in 227 KB of "
-                             "shared memory (split the group: fission/fusion plan)");
+                             "shared memory / 255 registers (split the group: fission/fusion plan)");
     L = best;
 }
 
@@ -570,6 +542,10 @@ void fill_report(const stencil_program *p, const Launch &L, sp_group_report *r) 
     r->bytes_exec = L.bytes_exec;
     r->flops_exec = L.flops_exec;
     r->smem_bytes_pt = L.smem_pt;
+    r->block_x = L.vx;
+    r->block_y = L.vy;
+    r->block_cby = L.cby;
+    r->t_model_us = L.t_model * 1e6;
     (void)p;
 }
 

@@ -30,7 +30,9 @@ struct ArrayDesc { std::string name; sp_role role; };
 struct Options {
     int fmad = 1;
     int tile_x = 0, tile_y = 0, zchunk = 0, threads = 0, prefetch = -1;
-    int loader = 0;  // 0: TMA + mbarrier ring, 1: cooperative ld.global -> st.shared
+    int loader = 0;
+    int block_x = 0, block_y = 0, block_cby = 0;  // register-block overrides (0 = chooser)
+    int zqueue = 1;  // 0: TMA + mbarrier ring, 1: cooperative ld.global -> st.shared
 };
 
 // ---------------------------------------------------------------- analysis
@@ -55,6 +57,7 @@ struct Stage {
     Keep keep = Keep::Dead;
     int cls = -1;           // region class (thread->point mapping)
     bool war_barrier = false;  // needs a CTA barrier before its store (R11 exception)
+    int sx0 = 0;            // smem layout left extension, ex0 rounded up to 16 B (vector alignment)
 };
 
 struct Input {
@@ -80,6 +83,8 @@ struct Launch {
     // configuration
     int tx = 0, ty = 0, zc = 0, nt = 0, pf = 0;
     int nth = 0;                 // threads per CTA (compute threads nt + producer warp)
+    int vx = 1, vy = 1, cby = 1; // register block of a thread: cby blocks of vx x vy core points
+    int zq = 1;                  // z-queues for values read at several planes
     int est_regs = 0;            // register estimate used by the tile chooser
     double t_model = 0;          // modelled launch time (s)
     int ntx = 0, nty = 0, nch = 0;
@@ -163,7 +168,9 @@ std::vector<std::vector<int>> greedy_plan(stencil_program *p);
 
 // codegen.cpp
 std::string generate_launch(const stencil_program *p, Launch &L, int index, bool fused);
-void core_geometry(const Launch &L, int *xt, int *yt, int *cpx, int *cpy);
+void core_geometry(const Launch &L, int *xt, int *yt);
+int codegen_regs(const stencil_program *p, const Launch &L);
+double codegen_smem_loads(const Launch &L);  // shared-memory loads per core point (all stages)
 
 // jit.cpp
 void compile_mode(stencil_program *p, Mode &m);

@@ -1,0 +1,98 @@
+"""z-slab decomposition on ONE GPU ("virtual ranks", test-only).
+
+Each rank is a Program over its slab (nz_global, z_offset, deep halo zhalo) with no
+communicator; before every fused group the test moves the ghost planes the library's
+exchange schedule names (sp_plan_exchange: arrays + depth) between the slab tensors
+with device-to-device copies — exactly the planes run_fused would ncclSend/ncclRecv.
+The P-rank result must equal the single-domain result bit for bit: initialisation is
+a function of global coordinates and the fused kernels recompute intermediates on
+deep-halo planes that are global interior (reading R1).
+"""
+import json
+import os
+
+import pytest
+
+from synth import programs as P
+from synth.fields import field_torch
+
+pytestmark = pytest.mark.gpu
+ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+
+
+def c4_small(nz):
+    from synth.scale_les import c4
+    prog = c4(nx=64, ny=32, nz=nz)
+    prog["plans"]["fused"] = json.load(open(os.path.join(ROOT, "configs", "c4_plan.json")))["groups"]
+    return prog
+
+
+def fill(p, prog, dev, z_offset, zhalo, nz_global=None):
+    hz = p.ghost[2]
+    nzl = p.n[2]
+    for aid, a in enumerate(prog["arrays"]):
+        v = field_torch(13, aid, p.n, p.ghost, prog["dtype"], dev, z_offset=z_offset,
+                        nz_alloc_extra=(zhalo - hz, zhalo - hz))
+        if nz_global is not None:
+            # no neighbour data before an exchange: poison deep-halo planes that are global interior
+            for pz in list(range(zhalo)) + list(range(zhalo + nzl, nzl + 2 * zhalo)):
+                if 0 <= z_offset - zhalo + pz < nz_global:  # x-y ghosts are physical (R1)
+                    hx, hy = p.ghost[0], p.ghost[1]
+                    v[pz, hy:hy + p.n[1], hx:hx + p.n[0]] = float("nan")
+        p.padded_view(p.tensors[a["name"]], hz=zhalo).copy_(v)
+
+
+def plane(p, t, z, depth):
+    """Planes [z, z+depth) (local interior coordinates) of an allocation."""
+    oz = p.layout["origin_z"]
+    return t[oz + z:oz + z + depth]
+
+
+@pytest.mark.parametrize("cfg,ranks", [("C2", 2), ("C5", 3), ("C3", 2), ("C4", 2), ("chain3", 3)])
+@pytest.mark.parametrize("fmad", [0, 1])
+def test_virtual_ranks_bitexact(cuda_device, cfg, ranks, fmad):
+    import torch
+    from paper_conf_hpdc_wahibm15_b200 import Program
+    nzl = 12
+    mk = {"C2": lambda nz: P.c2(nx=40, ny=24, nz=nz), "C5": lambda nz: P.c5(nx=32, ny=16, nz=nz),
+          "C3": lambda nz: P.c3(nx=48, ny=20, nz=nz), "C4": c4_small,
+          "chain3": lambda nz: P.resize(P.chain3(), 20, 12, nz)}[cfg]
+    glob = mk(nzl * ranks)
+    plan = glob["plans"]["fused"]
+    opts = {"fmad": fmad}
+    dev = cuda_device
+    # single domain
+    single = Program(glob, options=opts)
+    single.set_plan(plan)
+    single.allocate(dev)
+    fill(single, glob, dev, 0, glob["grid"]["ghost"][2])
+    single.run_fused()
+    # slabs
+    loc = mk(nzl)
+    probe = Program(loc, options=opts)
+    probe.set_plan(plan)
+    zhalo = max([max(r["z_below"], r["z_above"]) for r in probe.reports("fused")] +
+                [loc["grid"]["ghost"][2]])
+    slabs = []
+    for r in range(ranks):
+        s = Program(loc, nz_global=nzl * ranks, z_offset=r * nzl, zhalo=zhalo, options=opts)
+        s.set_plan(plan)
+        s.allocate(dev)
+        fill(s, loc, dev, r * nzl, zhalo, nz_global=nzl * ranks)
+        slabs.append(s)
+    for i in range(slabs[0].n_launches("fused")):
+        names, depth = slabs[0].exchange_plan("fused", i)
+        assert depth <= zhalo
+        for r in range(ranks - 1):  # r <-> r+1
+            lo, hi = slabs[r], slabs[r + 1]
+            for n in names:
+                plane(hi, hi.tensors[n], -depth, depth).copy_(plane(lo, lo.tensors[n], nzl - depth, depth))
+                plane(lo, lo.tensors[n], nzl, depth).copy_(plane(hi, hi.tensors[n], 0, depth))
+        for s in slabs:
+            s.run_launch("fused", i)
+    torch.cuda.synchronize()
+    outs = [a["name"] for a in glob["arrays"] if a["role"] in ("out", "inout")]
+    for n in outs:
+        want = single.interior_view(single.tensors[n])
+        got = torch.cat([s.interior_view(s.tensors[n]) for s in slabs], dim=0)
+        assert torch.equal(got, want), f"{cfg} {n}: slab result differs from single domain"

@@ -73,9 +73,16 @@ def test_parity_vs_oracle(cuda_device, name, prog, plans, fmad):
         assert_close(prog, got, ref, exact=exact)
 
 
-TILES = [dict(tile_x=16, tile_y=1, zchunk=1, threads=32), dict(tile_x=32, tile_y=4, zchunk=3),
-         dict(tile_x=64, tile_y=8, zchunk=7, threads=256, prefetch=1),
-         dict(tile_x=16, tile_y=16, zchunk=64, threads=512, prefetch=3)]
+# (tile, chunk, threads, prefetch, per-thread register block) combinations; the
+# register block geometry fixes tile_y = (threads / (tile_x / block_x)) * block_y * block_cby
+TILES = [dict(tile_x=16, tile_y=2, zchunk=1, threads=32, block_x=1, block_y=1, block_cby=1),
+         dict(tile_x=32, tile_y=4, zchunk=3, threads=64, block_x=2, block_y=1, block_cby=1),
+         dict(tile_x=64, tile_y=16, zchunk=7, threads=128, prefetch=1, block_x=2, block_y=2,
+              block_cby=2),
+         dict(tile_x=16, tile_y=16, zchunk=64, threads=64, prefetch=3, block_x=1, block_y=2,
+              block_cby=2),
+         dict(tile_x=64, tile_y=8, zchunk=5, threads=64, prefetch=2, block_x=4, block_y=2,
+              block_cby=1)]
 
 
 @pytest.mark.parametrize("tiles", TILES, ids=[str(i) for i in range(len(TILES))])

@@ -38,9 +38,23 @@ def load_workload(name):
         prog = c4()
         plan_path = os.path.join(ROOT, "configs", "c4_plan.json")
         if os.path.exists(plan_path):
-            prog["plans"]["fused"] = json.load(open(plan_path))["groups"]
+            pj = json.load(open(plan_path))
+            prog["plans"]["fused"] = pj["groups"]
+            prog["plan_configs"] = pj.get("configs")
         return prog
     return P.CONFIGS[name]()
+
+
+def tuned_configs(prog):
+    return prog.get("plan_configs")
+
+
+def apply_tuning(p, prog):
+    cfgs = tuned_configs(prog)
+    if cfgs:
+        for i, c in enumerate(cfgs):
+            if c:
+                p.tune("fused", i, c)
 
 
 def plan_of(prog):
@@ -141,12 +155,14 @@ def run_ours(args):
     # deep halo needed by the plan's accumulated z-reach (probe on the local grid)
     probe = Program(prog)
     probe.set_plan(plan)
+    apply_tuning(probe, prog)
     reach = max([max(r["z_below"], r["z_above"]) for r in probe.reports("fused")] + [prog["grid"]["ghost"][2]])
     zhalo = reach if world > 1 else prog["grid"]["ghost"][2]
     del probe
     comm = Comm(rank, world) if world > 1 else None
     p = Program(prog, comm=comm, nz_global=nz * world, z_offset=rank * nz, zhalo=zhalo)
     p.set_plan(plan)
+    apply_tuning(p, prog)
     p.allocate(dev, fill=0.0)
     fill_inputs(p, prog, dev, rank * nz, zhalo)
     stream = torch.cuda.current_stream(dev)

@@ -201,6 +201,20 @@ sp_status sp_plan_report(const stencil_program *prog, int32_t mode, int32_t laun
 sp_status fusion_plan_report(const stencil_program *prog, int32_t group, sp_group_report *out);
 /* Generated CUDA source of a mode (for inspection); *len receives the full size. */
 sp_status sp_plan_source(stencil_program *prog, int32_t mode, char *buf, size_t cap, size_t *len);
+/* Launch configuration (0 = left to the model-driven chooser).  The thread
+ * geometry must satisfy tile_x = (tile_x/block_x)*block_x and
+ * tile_y = (threads/(tile_x/block_x)) * block_y * block_cby. */
+typedef struct {
+    int32_t tile_x, tile_y, zchunk, threads, prefetch, block_x, block_y, block_cby;
+} sp_tile_config;
+
+/* Empirical tuning hook (the paper's per-kernel block-size tuning, §4.2):
+ * pin the configuration of one launch of a mode; cfg == NULL removes the pin.
+ * Re-analyses and regenerates the mode (JIT at the next compile/run).  Pins of
+ * the fused mode are dropped when a new plan is set.  SP_E_RESOURCES if the
+ * configuration does not fit. */
+sp_status sp_plan_tune(stencil_program *prog, int32_t mode, int32_t launch, const sp_tile_config *cfg);
+
 /* Halo-exchange schedule of one launch on several ranks: the arrays it reads
  * beyond the local slab (up to cap written to arrays[], *n = total) and the
  * exchange depth (its accumulated z reach, <= zhalo).  run_fused performs

@@ -15,7 +15,7 @@ import ctypes
 import os
 
 from ._abi import (SP_F32, SP_F64, ROLE, SpArrayDesc, SpEdge, SpGrid, SpGroupReport, SpKernel,
-                   SpLayout, SpStmt, SpStmtRef, SpTerm, SpTap, lib)
+                   SpLayout, SpStmt, SpStmtRef, SpTerm, SpTap, SpTileConfig, lib)
 
 __all__ = ["Program", "Comm", "StencilError", "lib"]
 
@@ -64,7 +64,10 @@ class Comm:
     def __del__(self):
         h = getattr(self, "handle", None)
         if h:
-            lib().sp_comm_destroy(h)
+            try:
+                lib().sp_comm_destroy(h)
+            except Exception:  # interpreter shutdown
+                pass
             self.handle = None
 
 
@@ -144,7 +147,10 @@ class Program:
     def __del__(self):
         h = getattr(self, "handle", None)
         if h:
-            lib().stencil_program_destroy(h)
+            try:
+                lib().stencil_program_destroy(h)
+            except Exception:  # interpreter shutdown
+                pass
             self.handle = None
 
     # ---------------------------------------------------------- memory
@@ -251,6 +257,15 @@ class Program:
         buf = ctypes.create_string_buffer(n.value + 1)
         _check(lib().sp_plan_source(self.handle, self._mode(mode), buf, n.value + 1, ctypes.byref(n)))
         return buf.value.decode()
+
+    def tune(self, mode, i, cfg):
+        """Pin launch i's configuration: dict with tile_x, tile_y, zchunk, threads, prefetch,
+        block_x, block_y, block_cby (missing/0 = chooser); None removes the pin."""
+        if cfg is None:
+            _check(lib().sp_plan_tune(self.handle, self._mode(mode), i, None))
+            return
+        c = SpTileConfig(**{k: int(v) for k, v in cfg.items() if k in dict(SpTileConfig._fields_)})
+        _check(lib().sp_plan_tune(self.handle, self._mode(mode), i, ctypes.byref(c)))
 
     def exchange_plan(self, mode, i):
         """(array names, depth) the executor exchanges before launch i on several ranks."""

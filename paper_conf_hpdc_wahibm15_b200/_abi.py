@@ -51,6 +51,11 @@ class SpLayout(ctypes.Structure):
                 ("bytes", ctypes.c_int64)]
 
 
+class SpTileConfig(ctypes.Structure):
+    _fields_ = [(n, ctypes.c_int32) for n in ("tile_x", "tile_y", "zchunk", "threads", "prefetch",
+                                              "block_x", "block_y", "block_cby")]
+
+
 class SpEdge(ctypes.Structure):
     _fields_ = [("frm", ctypes.c_int32), ("to", ctypes.c_int32), ("kind", ctypes.c_int32),
                 ("array", ctypes.c_int32)]
@@ -77,7 +82,7 @@ EXPORTS = [
     "stencil_program_destroy", "stencil_program_layout", "stencil_program_bind",
     "sp_program_set_option", "sp_program_counts", "sp_program_edges", "sp_fission_components",
     "fusion_plan_set", "sp_plan_greedy", "sp_plan_count", "sp_plan_report", "fusion_plan_report", "sp_plan_source",
-    "sp_plan_exchange", "sp_compile", "run_unfused", "run_fused", "sp_run_launch", "exchange_halos", "sp_last_error",
+    "sp_plan_exchange", "sp_plan_tune", "sp_compile", "run_unfused", "run_fused", "sp_run_launch", "exchange_halos", "sp_last_error",
 ]
 
 _lib = None
@@ -110,6 +115,7 @@ def lib():
             "sp_plan_source": [vp, i32, ctypes.c_char_p, ctypes.c_size_t, P(ctypes.c_size_t)],
             "sp_compile": [vp, i32],
             "sp_plan_exchange": [vp, i32, i32, i32, P(i32), P(i32), P(i32)],
+            "sp_plan_tune": [vp, i32, i32, P(SpTileConfig)],
             "run_unfused": [vp, vp],
             "run_fused": [vp, vp],
             "sp_run_launch": [vp, i32, i32, vp],

@@ -312,6 +312,32 @@ sp_status sp_plan_source(stencil_program *p, int32_t mode, char *buf, size_t cap
     });
 }
 
+sp_status sp_plan_tune(stencil_program *p, int32_t mode, int32_t launch, const sp_tile_config *cfg) {
+    return guard([&] {
+        if (!p) fail(SP_E_ARG, "null program");
+        Mode &m = mode_of(p, mode);
+        if (launch < 0 || launch >= (int)m.launches.size()) fail(SP_E_ARG, "launch index out of range");
+        auto &tune = mode ? p->tune_fused : p->tune_unfused;
+        auto saved = tune;
+        if (cfg) tune[launch] = *cfg;
+        else tune.erase(launch);
+        Mode n;
+        try {
+            if (mode) analyze_mode(p, true, p->plan_groups, n);
+            else {
+                std::vector<std::vector<int>> groups;
+                for (const Kernel &K : p->kernels) groups.push_back(K.stmts);
+                analyze_mode(p, false, groups, n);
+            }
+        } catch (...) {
+            tune = saved;
+            throw;
+        }
+        unload_mode(m);
+        m = std::move(n);
+    });
+}
+
 sp_status sp_plan_exchange(stencil_program *p, int32_t mode, int32_t launch, int32_t cap,
                            int32_t *arrays, int32_t *n, int32_t *depth) {
     return guard([&] {

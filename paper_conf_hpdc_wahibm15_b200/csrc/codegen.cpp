@@ -210,7 +210,7 @@ std::string generate_launch(const stencil_program *p, Launch &L, int index, bool
 
     // ------------------------------------------------------------ loads
     auto slot_of = [&](int a, const std::string &q) {
-        return "((" + q + " - (" + num(L.in[a].qlo) + ")) & " + num(L.in_depth[a] - 1) + ")";
+        return "((" + q + " - (" + num(L.in[a].qlo) + ")) % " + num(L.in_depth[a]) + ")";
     };
     auto box_bytes = [&](int a) { return (int64_t)L.in_rw[a] * L.in_rh[a] * p->elem; };
     auto issue_plane = [&](int a) {  // plane q of input a (variables q, bar in scope)
@@ -232,25 +232,28 @@ std::string generate_launch(const stencil_program *p, Launch &L, int index, bool
         }
         return s.str();
     };
-    // batch j: every input's plane j+ahi (and, for j == KF, all earlier planes from qlo)
+    // batch j: every input's plane j+ahi (and, for j == KF, all earlier planes from qlo);
+    // planes below an input's first needed plane qlo are never loaded
+    auto q0_of = [&](const Input &I) {
+        return "(j == KF) ? " + num(I.qlo) + " : max(j + (" + num(I.ahi) + "), " + num(I.qlo) + ")";
+    };
     auto batch = [&](std::ostringstream &s, const std::string &ind) {
         if (tma) {
             s << ind << "unsigned bytes = 0;\n";
             for (int a = 0; a < nin; ++a) {
                 const Input &I = L.in[a];
-                s << ind << "{ const int q0 = (j == KF) ? " << I.qlo << " : j + (" << I.ahi
-                  << "); const int q1 = min(j + (" << I.ahi << "), zc - 1 + (" << I.ahi
-                  << ")); if (q1 >= q0) bytes += (unsigned)(q1 - q0 + 1) * " << box_bytes(a)
-                  << "u; }\n";
+                s << ind << "{ const int q0 = " << q0_of(I) << "; const int q1 = min(j + (" << I.ahi
+                  << "), zc - 1 + (" << I.ahi << ")); if (q1 >= q0) bytes += (unsigned)(q1 - q0 + 1) * "
+                  << box_bytes(a) << "u; }\n";
             }
             s << ind << "sf_u64 *bar = &full[(j - KF) & " << NB - 1 << "];\n";
             s << ind << "sf_mbar_expect_tx(bar, bytes);\n";
         }
         for (int a = 0; a < nin; ++a) {
             const Input &I = L.in[a];
-            s << ind << "{ const int q0 = (j == KF) ? " << I.qlo << " : j + (" << I.ahi
-              << "); const int q1 = min(j + (" << I.ahi << "), zc - 1 + (" << I.ahi
-              << ")); for (int q = q0; q <= q1; ++q) " << issue_plane(a) << " }\n";
+            s << ind << "{ const int q0 = " << q0_of(I) << "; const int q1 = min(j + (" << I.ahi
+              << "), zc - 1 + (" << I.ahi << ")); for (int q = q0; q <= q1; ++q) " << issue_plane(a)
+              << " }\n";
         }
     };
 
@@ -404,8 +407,8 @@ std::string generate_launch(const stencil_program *p, Launch &L, int index, bool
         std::string slot;
         int64_t plane;
         if (l.stage) {
-            slot = "((k + (" + num(c) + ") - (" + num(L.st[l.id].loff) + ")) & " +
-                   num(L.st_depth[l.id] - 1) + ")";
+            slot = "((k + (" + num(c) + ") - (" + num(L.st[l.id].loff) + ")) % " +
+                   num(L.st_depth[l.id]) + ")";
             plane = L.st_plane[l.id];
         } else {
             slot = slot_of(l.id, "(k + (" + num(c) + "))");
@@ -643,9 +646,10 @@ std::string generate_launch(const stencil_program *p, Launch &L, int index, bool
             };
             o << "        #pragma unroll\n        for (int i = 0; i < " << hp[c] << "; ++i) {\n";
             o << "          const int f = h" << c << "_f[i];\n";
-            o << "          T v = " << term_expr(halo_operand) << ";\n";
-            o << "          if (!(zin && (f & 2))) v = sf_ldg_pred(gpl + h" << c
-              << "_g[i], zal && (f & 8));\n";
+            // ghost points (e.g. the y-halo rows of full-height tiles) are only loaded
+            o << "          T v;\n";
+            o << "          if (zin && (f & 2)) v = " << term_expr(halo_operand) << ";\n";
+            o << "          else v = sf_ldg_pred(gpl + h" << c << "_g[i], zal && (f & 8));\n";
             if (G.keep == Keep::Smem) {
                 Lay self{true, m};
                 o << "          " << bname(self, G.lead) << "[h" << c << "_" << lname(self)

@@ -232,7 +232,7 @@ static void layout_launch(const stencil_program *p, Launch &L) {
         int rw = (int)rup(L.tx + I.bx0 + std::max(I.ex1, 0), L.rw_pad);
         int rh = L.ty + I.ey0 + I.ey1;
         int64_t plane = rup((int64_t)rw * rh, 128 / e);
-        int D = pow2ceil(I.ahi - I.alo + 1 + L.pf);
+        int D = I.ahi - I.alo + 1 + L.pf;  // ring slot = plane mod D (constant modulo per step)
         L.in_off.push_back(off);
         L.in_plane.push_back(plane);
         L.in_rw.push_back(rw);
@@ -250,7 +250,7 @@ static void layout_launch(const stencil_program *p, Launch &L) {
         L.st_h.push_back(h);
         if (G.keep == Keep::Smem) {
             // one plane deeper than the reuse distance: no end-of-step barrier needed
-            int D = pow2ceil(G.depth + 1);
+            int D = G.depth + 1;
             int64_t plane = rup((int64_t)w * h, 128 / e);
             L.st_off.push_back(off);
             L.st_plane.push_back(plane);
@@ -503,7 +503,30 @@ void analyze_mode(stencil_program *p, bool fused, const std::vector<std::vector<
                                      std::to_string(std::max(L.z_below, L.z_above)) +
                                      " exceeds zhalo " + std::to_string(p->grid.zhalo));
         if (!L.dead) {
-            choose_config(p, L);
+            // per-launch tuned configuration (sp_plan_tune) overrides the chooser's search
+            auto &tune = fused ? p->tune_fused : p->tune_unfused;
+            auto it = tune.find((int)g);
+            if (it != tune.end()) {
+                Options saved = p->opt;
+                const sp_tile_config &c = it->second;
+                if (c.tile_x) p->opt.tile_x = c.tile_x;
+                if (c.tile_y) p->opt.tile_y = c.tile_y;
+                if (c.zchunk) p->opt.zchunk = c.zchunk;
+                if (c.threads) p->opt.threads = c.threads;
+                if (c.prefetch) p->opt.prefetch = c.prefetch;
+                if (c.block_x) p->opt.block_x = c.block_x;
+                if (c.block_y) p->opt.block_y = c.block_y;
+                if (c.block_cby) p->opt.block_cby = c.block_cby;
+                try {
+                    choose_config(p, L);
+                } catch (...) {
+                    p->opt = saved;
+                    throw;
+                }
+                p->opt = saved;
+            } else {
+                choose_config(p, L);
+            }
             model(p, L);
         }
         m.launches.push_back(std::move(L));
@@ -596,7 +619,14 @@ void sf_plan_set_impl(stencil_program *p, int32_t n_groups, const int32_t *group
                                       "') runs backwards in the plan");
         }
     Mode m;
-    analyze_mode(p, true, groups, m);  // throws on hazards / resources; old plan kept
+    auto saved_tune = p->tune_fused;
+    p->tune_fused.clear();  // tuned configurations belong to the previous plan
+    try {
+        analyze_mode(p, true, groups, m);  // throws on hazards / resources; old plan kept
+    } catch (...) {
+        p->tune_fused = saved_tune;
+        throw;
+    }
     unload_mode(p->fused);
     p->fused = std::move(m);
     p->plan_groups = groups;

@@ -32,7 +32,7 @@ struct Options {
     int tile_x = 0, tile_y = 0, zchunk = 0, threads = 0, prefetch = -1;
     int loader = 0;
     int block_x = 0, block_y = 0, block_cby = 0;  // register-block overrides (0 = chooser)
-    int zqueue = 1;  // 0: TMA + mbarrier ring, 1: cooperative ld.global -> st.shared
+    int zqueue = 0;  // z-queues cost registers/occupancy more than they save (measured r1)  // 0: TMA + mbarrier ring, 1: cooperative ld.global -> st.shared
 };
 
 // ---------------------------------------------------------------- analysis
@@ -84,7 +84,7 @@ struct Launch {
     int tx = 0, ty = 0, zc = 0, nt = 0, pf = 0;
     int nth = 0;                 // threads per CTA (compute threads nt + producer warp)
     int vx = 1, vy = 1, cby = 1; // register block of a thread: cby blocks of vx x vy core points
-    int zq = 1;                  // z-queues for values read at several planes
+    int zq = 0;                  // z-queues for values read at several planes
     int est_regs = 0;            // register estimate used by the tile chooser
     double t_model = 0;          // modelled launch time (s)
     int ntx = 0, nty = 0, nch = 0;
@@ -92,7 +92,7 @@ struct Launch {
     int rw_pad = 2;              // input row padding granularity (elements)
     // layout of smem (bytes) per input ring / stage ring
     std::vector<int64_t> in_off, in_plane;   // plane size in elements (padded)
-    std::vector<int> in_rw, in_rh, in_depth;  // ring depth: power of two
+    std::vector<int> in_rw, in_rh, in_depth;  // ring depth (planes)
     std::vector<int64_t> st_off, st_plane;
     std::vector<int> st_w, st_h, st_depth;
     int64_t bar_off = 0;
@@ -148,6 +148,7 @@ struct stencil_program_s {
     std::vector<std::vector<int>> plan_groups;  // gids per group
     int num_sms = 148;
     std::vector<void *> events;  // cudaEvent_t pool for exchange overlap
+    std::map<int, sp_tile_config> tune_fused, tune_unfused;  // sp_plan_tune overrides
 };
 
 namespace sf {

@@ -25,6 +25,7 @@ prog = bench.load_workload(a.workload)
 opts = {kv.split("=")[0]: int(kv.split("=")[1]) for kv in a.opt}
 p = Program(prog, options=opts)
 p.set_plan(bench.plan_of(prog))
+bench.apply_tuning(p, prog)
 dev = torch.device("cuda:0")
 p.allocate(dev, fill=0.0)
 bench.fill_inputs(p, prog, dev, 0, prog["grid"]["ghost"][2])

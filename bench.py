@@ -251,19 +251,57 @@ def run_ours(args):
     host_out = {n: torch.empty_like(p.tensors[n], device="cpu").pin_memory() for n in out_names}
     for n in in_names:
         host_in[n].copy_(p.tensors[n])
-    e2e_steps = max(1, min(args.steps, 10))
+    e2e_steps = max(2, min(args.steps, 10))
+    # Pipelined through the public API: step k's inputs go host->device on one copy
+    # stream and step k-1's outputs device->host on another while step k-1 computes;
+    # inputs and outputs are double-buffered and rebound (stencil_program_bind) per step.
+    dev_in = [{n: p.tensors[n] for n in in_names},
+              {n: torch.empty_like(p.tensors[n]) for n in in_names}]
+    dev_out = [{n: p.tensors[n] for n in out_names},
+               {n: dev_in[1][n] if n in in_names else torch.empty_like(p.tensors[n])
+                for n in out_names}]
+    for n in out_names:  # ghost cells of the second output buffer (never written by kernels)
+        if n not in in_names:
+            dev_out[1][n].copy_(p.tensors[n])
+    h2d_s, d2h_s = torch.cuda.Stream(dev), torch.cuda.Stream(dev)
+    in_ready = [torch.cuda.Event() for _ in range(e2e_steps)]
+    done = [torch.cuda.Event() for _ in range(e2e_steps)]
+    out_read = [torch.cuda.Event() for _ in range(e2e_steps)]
     barrier()
     s, e = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
     s.record(stream)
-    for _ in range(e2e_steps):
+    h2d_s.wait_event(s)
+    d2h_s.wait_event(s)
+    for k in range(e2e_steps):
+        b = k % 2
+        with torch.cuda.stream(h2d_s):
+            if k >= 2:
+                h2d_s.wait_event(done[k - 2])       # buffer b no longer read by step k-2
+            for n in in_names:
+                dev_in[b][n].copy_(host_in[n], non_blocking=True)
+            in_ready[k].record(h2d_s)
+        stream.wait_event(in_ready[k])
+        if k >= 2:
+            stream.wait_event(out_read[k - 2])       # outputs of step k-2 copied out
         for n in in_names:
-            p.tensors[n].copy_(host_in[n], non_blocking=True)
-        p.run_fused(stream)
+            p.bind(n, dev_in[b][n])
         for n in out_names:
-            host_out[n].copy_(p.tensors[n], non_blocking=True)
+            p.bind(n, dev_out[b][n])
+        p.run_fused(stream)
+        done[k].record(stream)
+        with torch.cuda.stream(d2h_s):
+            d2h_s.wait_event(done[k])
+            for n in out_names:
+                host_out[n].copy_(dev_out[b][n], non_blocking=True)
+            out_read[k].record(d2h_s)
+    stream.wait_event(out_read[e2e_steps - 1])
     e.record(stream)
     barrier()
     e2e_ms = max_over_ranks(s.elapsed_time(e) / e2e_steps)
+    for n in in_names:
+        p.bind(n, dev_in[0][n])
+    for n in out_names:
+        p.bind(n, dev_out[0][n])
     h2d = sum(host_in[n].numel() * host_in[n].element_size() for n in in_names)
     d2h = sum(host_out[n].numel() * host_out[n].element_size() for n in out_names)
 

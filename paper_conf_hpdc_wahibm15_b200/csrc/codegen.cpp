@@ -550,8 +550,13 @@ std::string generate_launch(const stencil_program *p, Launch &L, int index, bool
             if (pi.cmax > pi.cmin) return qname(m, k) + "[b][" + num(cc - pi.cmin) + "]";
             return dname(s.stage, s.idx, cc, k.y, k.x);
         };
+        // Parity build (fmad=0): one left-to-right sum, the fixed order of R4 (bit-exact
+        // with the oracle).  Perf build: ACC interleaved partial sums (term t goes to sum
+        // t % ACC) added at the end — independent FMA chains for ILP; the reassociation
+        // is within the 1e-12 / 1e-5 tolerance like the FMA contraction itself.
+        const int ACC = (p->opt.fmad && G.terms.size() >= 6) ? p->opt.acc_split : 1;
         auto term_expr = [&](const std::function<std::string(const Src &)> &opd) {
-            std::string e;
+            std::vector<std::string> part(ACC);
             for (size_t ti = 0; ti < G.terms.size(); ++ti) {
                 const TermR &t = G.terms[ti];
                 std::string a = opd(t.a);
@@ -560,8 +565,11 @@ std::string generate_launch(const stencil_program *p, Launch &L, int index, bool
                 else if (t.coef == -1.0) term = "(-" + a + ")";
                 else term = "(T)" + lit(t.coef, f32) + " * " + a;
                 if (t.has_b) term = "(" + term + ") * " + opd(t.b);
-                e = ti == 0 ? term : "(" + e + ") + " + term;
+                std::string &e = part[ti % ACC];
+                e = e.empty() ? term : "(" + e + ") + " + term;
             }
+            std::string e = part[0];
+            for (int a = 1; a < ACC; ++a) e = "(" + e + ") + (" + part[a] + ")";
             return e;
         };
         for (int iy = 0; iy < VY; ++iy)

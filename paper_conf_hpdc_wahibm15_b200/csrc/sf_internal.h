@@ -32,7 +32,8 @@ struct Options {
     int tile_x = 0, tile_y = 0, zchunk = 0, threads = 0, prefetch = -1;
     int loader = 0;
     int block_x = 0, block_y = 0, block_cby = 0;  // register-block overrides (0 = chooser)
-    int zqueue = 0;  // z-queues cost registers/occupancy more than they save (measured r1)  // 0: TMA + mbarrier ring, 1: cooperative ld.global -> st.shared
+    int zqueue = 0;  // z-queues cost registers/occupancy more than they save (measured r1)
+    int acc_split = 1;  // >1: interleaved partial sums in the perf build (no gain measured r1)  // 0: TMA + mbarrier ring, 1: cooperative ld.global -> st.shared
 };
 
 // ---------------------------------------------------------------- analysis

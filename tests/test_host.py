@@ -247,3 +247,56 @@ def test_generated_kernels_compile_for_sm100a(name):
             for r in p.reports("fused"):
                 assert 0 < r["regs_per_thread"] <= 255
                 assert r["smem_bytes"] <= 227 * 1024
+
+
+# ----------------------------------------------------------------- tuning / exchange / planner
+def test_plan_tune_pins_and_resets():
+    prog = P.c2(n=64)
+    p = Program(prog)
+    p.set_plan(prog["plans"]["fused"])
+    cfg = dict(tile_x=64, tile_y=8, threads=128, block_x=1, block_y=4, block_cby=1, zchunk=16)
+    p.tune("fused", 0, cfg)
+    r = p.report("fused", 0)
+    assert (r["tile_x"], r["tile_y"], r["threads"], r["block_y"], r["zchunk"]) == (64, 8, 128, 4, 16)
+    p.tune("fused", 0, None)
+    assert p.report("fused", 0)["tile_y"] != 8 or p.report("fused", 0)["zchunk"] != 16
+    with pytest.raises(StencilError) as e:   # inconsistent thread geometry
+        p.tune("fused", 0, dict(tile_x=64, tile_y=3, threads=128, block_x=1, block_y=1, block_cby=1))
+    assert e.value.code == 6
+    p.tune("fused", 0, cfg)
+    p.set_plan(prog["plans"]["fused"])      # a new plan drops the pins
+    assert p.report("fused", 0)["zchunk"] != 16 or p.report("fused", 0)["tile_y"] != 8
+
+
+def test_exchange_schedule_matches_reach():
+    prog = P.c3(n=32)
+    p = Program(prog, nz_global=64, z_offset=0, zhalo=5)
+    p.set_plan(prog["plans"]["fission_fused"])
+    names, depth = p.exchange_plan("fused", 0)
+    assert names == ["A"] and depth == 5          # 7pt, 7pt, 13pt, 7pt chain: reach 1+1+2+1
+    names, depth = p.exchange_plan("fused", 1)
+    assert names == ["B"] and depth == 5          # O1 is read point-wise: no exchange
+    u_names, u_depth = p.exchange_plan("unfused", 2)
+    assert u_names == ["P1"] and u_depth == 2     # the 13-point kernel alone
+
+
+def test_deep_halo_must_cover_reach():
+    prog = P.c3(n=32)
+    p = Program(prog, nz_global=64, z_offset=0, zhalo=4)
+    p.set_plan(prog["plans"]["unfused"])          # reach <= 2: fine
+    # single-rank programs do not exchange, so any reach is allowed there
+    q = Program(prog, zhalo=2)
+    q.set_plan(prog["plans"]["single"])
+
+
+def test_greedy_plan_is_legal_and_reduces_traffic():
+    from synth.scale_les import c4
+    prog = c4(nx=256, ny=32, nz=64)
+    p = Program(prog)
+    plan = p.plan_greedy()
+    p.set_plan(plan)
+    fused = sum(r["bytes_alg"] for r in p.reports("fused"))
+    unfused = sum(r["bytes_alg"] for r in p.reports("unfused"))
+    assert fused < 0.7 * unfused
+    refs = [r for g in plan for r in g]
+    assert len(refs) == len(set(refs)) == sum(len(k["stmts"]) for k in prog["kernels"])

@@ -94,36 +94,57 @@ class Timer:
         sub["plans"] = {"fused": [[k["name"] for k in kernels]]}
         return sub
 
+    def _timeit(self, p):
+        p.run_launch("fused", 0)
+        torch.cuda.synchronize()
+        ts = []
+        for _ in range(self.iters):
+            self.flush.zero_()
+            s, e = torch.cuda.Event(True), torch.cuda.Event(True)
+            s.record()
+            p.run_launch("fused", 0)
+            e.record()
+            torch.cuda.synchronize()
+            ts.append(s.elapsed_time(e) * 1e-3)
+        return sorted(ts)[len(ts) // 2]
+
     def time(self, refs):
+        """Measured time of a candidate group: the chooser's configuration and the
+        hint configurations (winners of earlier tuning), best of them."""
         key = tuple(sorted(refs, key=lambda r: self.pos[r]))
         if key in self.cache:
             return self.cache[key]
         sub = self.subprogram(key)
+        t = float("inf")
         try:
             p = Program(sub)
             p.set_plan(sub["plans"]["fused"])
             for a in sub["arrays"]:
                 p.bind(a["name"], self.tensors[a["name"]])
-            p.run_launch("fused", 0)
-            torch.cuda.synchronize()
-            ts = []
-            for _ in range(self.iters):
-                self.flush.zero_()
-                s, e = torch.cuda.Event(True), torch.cuda.Event(True)
-                s.record()
-                p.run_launch("fused", 0)
-                e.record()
-                torch.cuda.synchronize()
-                ts.append(s.elapsed_time(e) * 1e-3)
-            t = sorted(ts)[len(ts) // 2]
+            t = self._timeit(p)
+            for cfg in self.hints:
+                try:
+                    p.tune("fused", 0, cfg)
+                    t = min(t, self._timeit(p))
+                except StencilError:
+                    pass
         except StencilError:
-            t = float("inf")
+            pass
         self.cache[key] = t
         return t
 
+    hints = []
 
-def autotune(prog, log=print, max_group=64):
+
+HINTS_F64 = [dict(tile_x=64, tile_y=4, threads=128, block_x=1, block_y=2, block_cby=1, zchunk=32),
+             dict(tile_x=32, tile_y=8, threads=128, block_x=1, block_y=2, block_cby=1, zchunk=32),
+             dict(tile_x=32, tile_y=8, threads=256, block_x=1, block_y=1, block_cby=1, zchunk=32)]
+
+
+def autotune(prog, log=print, max_group=64, hints=True):
     T = Timer(prog)
+    if hints and prog["dtype"] == "f64":
+        T.hints = HINTS_F64
     full = T._full
     groups = []
     for k in prog["kernels"]:
@@ -158,15 +179,17 @@ def config_candidates(prog):
     out = []
     for tx in tiles:
         for nt in (128, 256):
-            for bx, by, cb in ((1, 1, 1), (1, 2, 1), (2, 2, 1), (1, 1, 2)):
+            for bx, by, cb in ((1, 1, 1), (1, 2, 1), (2, 2, 1), (1, 1, 2), (1, 4, 1), (1, 2, 2),
+                               (2, 2, 2), (1, 4, 2)):
                 xt = tx // bx
-                if nt % xt or xt > nt:
+                if nt % xt or xt > nt or bx * by * cb > 8:
                     continue
                 ty = nt // xt * by * cb
                 if ty > 32 or ty > 2 * ny:
                     continue
+                # tall tiles have fewer CTAs: give them shorter z-chunks
                 out.append(dict(tile_x=tx, tile_y=ty, threads=nt, block_x=bx, block_y=by,
-                                block_cby=cb, zchunk=32))
+                                block_cby=cb, zchunk=32 if ty < 16 else 16))
     return out
 
 
@@ -206,15 +229,20 @@ def tune_configs(prog, groups, tensors, log=print, iters=7):
             if t < best:
                 best, bcfg = t, cfg
         if bcfg is not None:
-            for zc in (16, 64):
-                cfg = dict(bcfg, zchunk=zc)
-                try:
-                    p.tune("fused", i, cfg)
-                    t = timeit(i)
-                except StencilError:
-                    continue
-                if t < best:
-                    best, bcfg = t, cfg
+            # refine around the winner: z-chunk, then TMA prefetch distance
+            for key, values in (("zchunk", (16, 64)), ("prefetch", (1, 2, 3))):
+                base = bcfg
+                for v in values:
+                    cfg = dict(base, **{key: v})
+                    if cfg == base:
+                        continue
+                    try:
+                        p.tune("fused", i, cfg)
+                        t = timeit(i)
+                    except StencilError:
+                        continue
+                    if t < best:
+                        best, bcfg = t, cfg
         p.tune("fused", i, bcfg)
         best_cfgs.append(bcfg)
         log(f"group {i}: {best*1e6:.1f} us with {bcfg or 'chooser'}")

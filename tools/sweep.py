@@ -28,6 +28,7 @@ def main():
     ap.add_argument("--grid", action="store_true", help="enumerate tile/block combinations")
     ap.add_argument("--zchunk", type=int, default=32)
     ap.add_argument("--tx", default="32,64")
+    ap.add_argument("--apply-tuning", action="store_true", help="pin the plan's tuned configs first")
     a = ap.parse_args()
     if a.grid:
         for tx in [int(v) for v in a.tx.split(",")]:
@@ -58,6 +59,8 @@ def main():
             p = Program(prog, options=opts)
             if a.mode == "fused":
                 p.set_plan(plan)
+                if a.apply_tuning:
+                    bench.apply_tuning(p, prog)
             if base is None:
                 p.allocate(dev, fill=0.0)
                 bench.fill_inputs(p, prog, dev, 0, prog["grid"]["ghost"][2])

@@ -192,45 +192,35 @@ def run_ours(args):
     sampler.start()
     time.sleep(0.25)
     per_launch = [0.0] * len(reps_f)
-    if world == 1:
-        # events between launches: per-launch durations on the launching stream
-        evs = [[torch.cuda.Event(enable_timing=True) for _ in range(len(live_f) + 1)]
-               for _ in range(args.steps)]
-        barrier()
-        t0 = time.perf_counter()
-        for k in range(args.steps):
-            for j, i in enumerate(live_f):
-                evs[k][j].record(stream)
-                p.run_launch("fused", i, stream)
-            evs[k][-1].record(stream)
-        barrier()
-        wall = time.perf_counter() - t0
-        step_ms = sum(evs[k][0].elapsed_time(evs[k][-1]) for k in range(args.steps)) / args.steps
-        for j, i in enumerate(live_f):
-            per_launch[i] = sum(evs[k][j].elapsed_time(evs[k][j + 1])
-                                for k in range(args.steps)) / args.steps
-    else:
-        s, e = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
-        barrier()
-        t0 = time.perf_counter()
-        s.record(stream)
-        for k in range(args.steps):
-            p.run_fused(stream)
-        e.record(stream)
-        barrier()
-        wall = time.perf_counter() - t0
-        step_ms = s.elapsed_time(e) / args.steps
+    # headline: K steps back to back (launches adjacent on the stream, so programmatic
+    # dependent launch overlaps each group's prologue with the previous group's tail)
+    s, e = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+    barrier()
+    t0 = time.perf_counter()
+    s.record(stream)
+    for k in range(args.steps):
+        p.run_fused(stream)
+    e.record(stream)
+    barrier()
+    wall = time.perf_counter() - t0
+    step_ms = s.elapsed_time(e) / args.steps
     clocks = sampler.stop()
     step_ms = max_over_ranks(step_ms)
-    if world > 1:  # per-launch durations from a separate pass (no exchange)
-        for i in live_f:
-            s, e = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
-            s.record(stream)
-            for _ in range(10):
-                p.run_launch("fused", i, stream)
-            e.record(stream)
-            torch.cuda.synchronize(dev)
-            per_launch[i] = s.elapsed_time(e) / 10
+    # per-launch durations (dominant kernel of the roofline): a second timed pass of
+    # the same launches with CUDA events between them on the launching stream
+    prof_steps = max(3, min(args.steps, 50))
+    evs = [[torch.cuda.Event(enable_timing=True) for _ in range(len(live_f) + 1)]
+           for _ in range(prof_steps)]
+    barrier()
+    for k in range(prof_steps):
+        for j, i in enumerate(live_f):
+            evs[k][j].record(stream)
+            p.run_launch("fused", i, stream)
+        evs[k][-1].record(stream)
+    barrier()
+    for j, i in enumerate(live_f):
+        per_launch[i] = sum(evs[k][j].elapsed_time(evs[k][j + 1])
+                            for k in range(prof_steps)) / prof_steps
 
     # ---------------------------------------------------------- unfused, same K
     for _ in range(args.warmup):

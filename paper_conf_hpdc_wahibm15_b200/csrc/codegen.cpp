@@ -266,9 +266,12 @@ std::string generate_launch(const stencil_program *p, Launch &L, int index, bool
         for (int a = 0; a < nin; ++a) o << "    sf_prefetch_tmap(&p.tm[" << a << "]);\n";
     }
     o << "  }\n  __syncthreads();\n";
+    const bool pdl = p->opt.pdl != 0;
+    if (pdl) o << "  sf_pdl_launch_dependents();  // the next group may start its prologue\n";
     if (tma) {
         o << "  if (tid >= NT) {  // ---- TMA producer warp: batch j for step j, PF steps ahead\n";
         o << "    if (tid == NT) {\n";
+        if (pdl) o << "      sf_pdl_wait();  // inputs written by the previous group are complete\n";
         o << "      for (int j = KF; j < zc; ++j) {\n";
         o << "        const int s = j - 1 - PF;  // step whose slots batch j overwrites\n";
         o << "        if (s >= KF) sf_mbar_wait(&empty[(s - KF) & " << NE - 1 << "], ((s - KF) >> "
@@ -276,6 +279,9 @@ std::string generate_launch(const stencil_program *p, Launch &L, int index, bool
         batch(o, "        ");
         o << "      }\n    }\n    return;\n  }\n";
     }
+    // compute warps store arrays the previous group may still read (WAR) and read
+    // what it wrote: wait for its completion before any global access
+    if (pdl) o << "  sf_pdl_wait();\n";
 
     // ---------------------------------------------------- layouts
     struct Lay {

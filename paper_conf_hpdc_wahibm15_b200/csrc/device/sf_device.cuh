@@ -59,6 +59,13 @@ __device__ __forceinline__ void sf_bar_sync(int id, int nthreads) {
     asm volatile("bar.sync %0, %1;" ::"r"(id), "r"(nthreads) : "memory");
 }
 
+// programmatic dependent launch: let the next group's grid start its prologue, and
+// wait for the previous grid's memory operations before touching dependent data
+__device__ __forceinline__ void sf_pdl_launch_dependents() {
+    asm volatile("griddepcontrol.launch_dependents;" ::: "memory");
+}
+__device__ __forceinline__ void sf_pdl_wait() { asm volatile("griddepcontrol.wait;" ::: "memory"); }
+
 __device__ __forceinline__ void sf_prefetch_tmap(const SfTmap *m) {
     asm volatile("prefetch.tensormap [%0];" ::"l"(m) : "memory");
 }

@@ -41,6 +41,7 @@ struct Drv {
                                      CUtensorMapSwizzle, CUtensorMapL2promotion,
                                      CUtensorMapFloatOOBfill) = nullptr;
     CUresult (*GetErrorString)(CUresult, const char **) = nullptr;
+    CUresult (*LaunchKernelEx)(const CUlaunchConfig *, CUfunction, void **, void **) = nullptr;
     bool ok = false;
 };
 static Drv g_drv;
@@ -86,6 +87,7 @@ void ensure_cuda() {
     entry("cuLaunchKernel", g_drv.LaunchKernel);
     entry("cuTensorMapEncodeTiled", g_drv.TensorMapEncodeTiled);
     entry("cuGetErrorString", g_drv.GetErrorString);
+    entry("cuLaunchKernelEx", g_drv.LaunchKernelEx);
     g_drv.ok = true;
 }
 
@@ -262,6 +264,27 @@ void launch(stencil_program *p, Mode &m, int i, void *stream, int chunk_first, i
     int32_t ints[2] = {chunk_first, chunk_step};
     std::memcpy(base + L.int_off, ints, 8);
     void *args[] = {base};
+    if (p->opt.pdl) {
+        // programmatic dependent launch: the kernel's prologue may overlap the previous
+        // launch on the stream; griddepcontrol.wait in the kernel orders its data accesses
+        CUlaunchAttribute attr[1];
+        std::memset(attr, 0, sizeof attr);
+        attr[0].id = CU_LAUNCH_ATTRIBUTE_PROGRAMMATIC_STREAM_SERIALIZATION;
+        attr[0].value.programmaticStreamSerializationAllowed = 1;
+        CUlaunchConfig cfg;
+        std::memset(&cfg, 0, sizeof cfg);
+        cfg.gridDimX = (unsigned)L.ntx;
+        cfg.gridDimY = (unsigned)L.nty;
+        cfg.gridDimZ = (unsigned)nchunks;
+        cfg.blockDimX = (unsigned)L.nth;
+        cfg.blockDimY = cfg.blockDimZ = 1;
+        cfg.sharedMemBytes = (unsigned)L.smem;
+        cfg.hStream = (CUstream)stream;
+        cfg.attrs = attr;
+        cfg.numAttrs = 1;
+        drv_check(g_drv.LaunchKernelEx(&cfg, (CUfunction)L.func, args, nullptr), "cuLaunchKernelEx");
+        return;
+    }
     drv_check(g_drv.LaunchKernel((CUfunction)L.func, (unsigned)L.ntx, (unsigned)L.nty,
                                  (unsigned)nchunks, (unsigned)L.nth, 1, 1, (unsigned)L.smem,
                                  (CUstream)stream, args, nullptr),

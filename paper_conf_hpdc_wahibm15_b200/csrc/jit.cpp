@@ -264,7 +264,7 @@ void launch(stencil_program *p, Mode &m, int i, void *stream, int chunk_first, i
     int32_t ints[2] = {chunk_first, chunk_step};
     std::memcpy(base + L.int_off, ints, 8);
     void *args[] = {base};
-    if (p->opt.pdl) {
+    if (L.pdl) {
         // programmatic dependent launch: the kernel's prologue may overlap the previous
         // launch on the stream; griddepcontrol.wait in the kernel orders its data accesses
         CUlaunchAttribute attr[1];

@@ -33,7 +33,7 @@ struct Options {
     int loader = 0;
     int block_x = 0, block_y = 0, block_cby = 0;  // register-block overrides (0 = chooser)
     int zqueue = 0;  // z-queues cost registers/occupancy more than they save (measured r1)
-    int pdl = 1;        // programmatic dependent launch between consecutive launches
+    int pdl = 1;        // programmatic dependent launch: 1 = fused groups, 2 = all, 0 = off
     int acc_split = 1;  // >1: interleaved partial sums in the perf build (no gain measured r1)  // 0: TMA + mbarrier ring, 1: cooperative ld.global -> st.shared
 };
 
@@ -111,6 +111,7 @@ struct Launch {
     void *module = nullptr;  // CUmodule
     size_t param_size = 0, ptr_off = 0, int_off = 0;
     bool dead = false;       // nothing to compute (all stages dead)
+    bool pdl = false;        // launched with programmatic stream serialization
 };
 
 struct Mode {

@@ -202,6 +202,9 @@ sp_status sp_program_set_option(stencil_program *p, const char *key, int64_t v) 
         else if (k == "block_y") o.block_y = (int)v;
         else if (k == "block_cby") o.block_cby = (int)v;
         else if (k == "zqueue") o.zqueue = (int)v;
+        else if (k == "suspend_hint") o.suspend_hint = (int)v;
+        else if (k == "coef_const") o.coef_const = (int)v;
+        else if (k == "l2pf") o.l2pf = (int)v;
         else if (k == "pdl") o.pdl = std::max(0, std::min(2, (int)v));
         else if (k == "acc_split") o.acc_split = std::max(1, std::min(4, (int)v));
         else if (k == "l2_flush") {}

@@ -29,6 +29,7 @@
 // array's ghost value through a predicated load; tiles inside the interior skip
 // the test.
 #include <cstdio>
+#include <cstring>
 #include <functional>
 #include <set>
 #include <sstream>
@@ -166,7 +167,8 @@ std::string generate_launch(const stencil_program *p, Launch &L, int index, bool
     const int NB = L.nbar_full, NE = L.nbar_empty;
 
     o << "// generated by stencilfuse codegen: " << (fused ? "fused group " : "original kernel ")
-      << L.name << "\n#include \"sf_device.cuh\"\n";
+      << L.name << "\n#define SF_SUSPEND_HINT " << p->opt.suspend_hint
+      << "\n#include \"sf_device.cuh\"\n";
     o << "namespace " << L.fn << "_ns {\n";
     o << "typedef " << T << " T;\ntypedef " << T2 << " T2;\n";
     o << "constexpr int TX = " << L.tx << ", TY = " << L.ty << ", NT = " << L.nt << ", ZC = " << L.zc
@@ -182,7 +184,22 @@ std::string generate_launch(const stencil_program *p, Launch &L, int index, bool
     o << "struct __align__(64) Params { SfTmap tm[" << std::max(nin, 1) << "]; T *arr["
       << std::max(narr, 1) << "]; int chunk_first, chunk_step; };\n";
     o << "static_assert(sizeof(SfTmap) * " << std::max(nin, 1) << " == " << L.ptr_off
-      << ", \"param layout\");\n}\n";
+      << ", \"param layout\");\n";
+    // statement coefficients live in constant memory: FP64 FMA/MUL take them as
+    // constant-bank operands instead of re-materialising each one per use
+    o << "/*SF_COEF_TABLE*/\n}\n";
+    std::map<uint64_t, int> coef_idx;
+    std::vector<double> coefs;
+    auto coef_ref = [&](double c) {
+        uint64_t bits;
+        std::memcpy(&bits, &c, 8);
+        auto it = coef_idx.find(bits);
+        if (it == coef_idx.end()) {
+            it = coef_idx.emplace(bits, (int)coefs.size()).first;
+            coefs.push_back(c);
+        }
+        return "SFK[" + num(it->second) + "]";
+    };
     o << "extern \"C\" __global__ void __launch_bounds__(" << L.nth << ", 1) " << L.fn
       << "(const __grid_constant__ " << L.fn << "_ns::Params p) {\n";
     o << "  using namespace " << L.fn << "_ns;\n";
@@ -275,7 +292,24 @@ std::string generate_launch(const stencil_program *p, Launch &L, int index, bool
         o << "  if (tid >= NT) {  // ---- TMA producer warp: batch j for step j, PF steps ahead\n";
         o << "    if (tid == NT) {\n";
         if (pdl) o << "      sf_pdl_wait();  // inputs written by the previous group are complete\n";
+        const int L2PF = p->opt.l2pf;
+        auto l2_prefetch = [&](const std::string &jexpr, const std::string &ind) {
+            // the plane batch `jexpr` will load, prefetched into L2 (independent of the ring)
+            for (int a = 0; a < nin; ++a) {
+                const Input &I = L.in[a];
+                o << ind << "{ const int q = " << jexpr << " + (" << I.ahi << "); if (q >= " << I.qlo
+                  << " && q <= zc - 1 + (" << I.ahi << ")) sf_tma_prefetch_3d(&p.tm[" << a
+                  << "], X0 + (" << -I.bx0 << ") + OXA, Y0 + (" << -I.ey0
+                  << ") + OYA, Z0 + q + OZA); }\n";
+            }
+        };
+        if (L2PF > 0) {
+            o << "      for (int j = KF + 1; j < min(KF + " << L2PF << ", zc); ++j) {\n";
+            l2_prefetch("j", "        ");
+            o << "      }\n";
+        }
         o << "      for (int j = KF; j < zc; ++j) {\n";
+        if (L2PF > 0) l2_prefetch("(j + " + num(L2PF) + ")", "        ");
         o << "        const int s = j - 1 - PF;  // step whose slots batch j overwrites\n";
         o << "        if (s >= KF) sf_mbar_wait(&empty[(s - KF) & " << NE - 1 << "], ((s - KF) >> "
           << log2i(NE) << ") & 1);\n";
@@ -572,7 +606,8 @@ std::string generate_launch(const stencil_program *p, Launch &L, int index, bool
                 std::string term;
                 if (t.coef == 1.0) term = a;
                 else if (t.coef == -1.0) term = "(-" + a + ")";
-                else term = "(T)" + lit(t.coef, f32) + " * " + a;
+                else term = (p->opt.coef_const ? coef_ref(t.coef) : "(T)" + lit(t.coef, f32)) +
+                            " * " + a;
                 if (t.has_b) term = "(" + term + ") * " + opd(t.b);
                 std::string &e = part[ti % ACC];
                 e = e.empty() ? term : "(" + e + ") + " + term;
@@ -687,6 +722,13 @@ std::string generate_launch(const stencil_program *p, Launch &L, int index, bool
     }
     o << "  }\n}\n";
     L.source = o.str();
+    std::ostringstream tbl;
+    tbl << "__constant__ T SFK[" << std::max<size_t>(coefs.size(), 1) << "] = {";
+    for (size_t i = 0; i < coefs.size(); ++i) tbl << (i ? ", " : "") << lit(coefs[i], f32);
+    if (coefs.empty()) tbl << "0";
+    tbl << "};";
+    const std::string marker = "/*SF_COEF_TABLE*/";
+    L.source.replace(L.source.find(marker), marker.size(), tbl.str());
     return L.source;
 }
 

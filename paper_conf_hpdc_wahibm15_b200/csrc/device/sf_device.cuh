@@ -39,7 +39,22 @@ __device__ __forceinline__ void sf_mbar_expect_tx(sf_u64 *bar, sf_u32 bytes) {
                  : "memory");
 }
 
+// Phase-parity wait.  SF_SUSPEND_HINT (ns, per generated kernel) adds a suspend-time
+// hint to try_wait so a waiting warp may sleep instead of re-issuing the test; off by
+// default (a large hint slowed the C4 step by 35 % in round 1 measurements).
+#ifndef SF_SUSPEND_HINT
+#define SF_SUSPEND_HINT 0
+#endif
 __device__ __forceinline__ void sf_mbar_wait(sf_u64 *bar, sf_u32 parity) {
+#if SF_SUSPEND_HINT
+    asm volatile(
+        "{\n\t.reg .pred P1;\n"
+        "SF_WAIT_%=:\n\t"
+        "mbarrier.try_wait.parity.shared::cta.b64 P1, [%0], %1, %2;\n\t"
+        "@!P1 bra SF_WAIT_%=;\n}" ::"r"(sf_smem_addr(bar)),
+        "r"(parity), "r"(SF_SUSPEND_HINT)
+        : "memory");
+#else
     asm volatile(
         "{\n\t.reg .pred P1;\n"
         "SF_WAIT_%=:\n\t"
@@ -47,6 +62,7 @@ __device__ __forceinline__ void sf_mbar_wait(sf_u64 *bar, sf_u32 parity) {
         "@!P1 bra SF_WAIT_%=;\n}" ::"r"(sf_smem_addr(bar)),
         "r"(parity)
         : "memory");
+#endif
 }
 
 // consumer release of a ring slot (default .release.cta semantics)
@@ -78,6 +94,15 @@ __device__ __forceinline__ void sf_tma_load_3d(void *dst, const SfTmap *map, sf_
         "cp.async.bulk.tensor.3d.shared::cluster.global.tile.mbarrier::complete_tx::bytes"
         " [%0], [%1, {%3, %4, %5}], [%2];" ::"r"(sf_smem_addr(dst)),
         "l"(map), "r"(sf_smem_addr(bar)), "r"(x), "r"(y), "r"(z)
+        : "memory");
+}
+
+// L2 prefetch of a plane box (no shared memory, no completion): raises the DRAM
+// requests in flight beyond what the shared-memory rings can hold
+__device__ __forceinline__ void sf_tma_prefetch_3d(const SfTmap *map, int x, int y, int z) {
+    asm volatile(
+        "cp.async.bulk.prefetch.tensor.3d.L2.global.tile [%0, {%1, %2, %3}];" ::"l"(map), "r"(x),
+        "r"(y), "r"(z)
         : "memory");
 }
 

@@ -36,7 +36,8 @@ def load_workload(name):
     if name == "C4":
         from synth.scale_les import c4
         prog = c4()
-        plan_path = os.path.join(ROOT, "configs", "c4_plan.json")
+        # SF_C4_PLAN: candidate plan file for A/B runs (dev tools); default the frozen plan
+        plan_path = os.environ.get("SF_C4_PLAN") or os.path.join(ROOT, "configs", "c4_plan.json")
         if os.path.exists(plan_path):
             pj = json.load(open(plan_path))
             prog["plans"]["fused"] = pj["groups"]
@@ -409,7 +410,7 @@ def run_reference(args):
 def main():
     ap = argparse.ArgumentParser()
     ap.add_argument("--gpus", type=int, default=1)
-    ap.add_argument("--steps", type=int, default=500)
+    ap.add_argument("--steps", type=int, default=200)
     ap.add_argument("--warmup", type=int, default=10)
     ap.add_argument("--workload", default="C4", choices=["C1", "C2", "C3", "C4", "C5"])
     ap.add_argument("--impl", default="ours", choices=["ours", "reference"])

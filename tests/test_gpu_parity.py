@@ -116,6 +116,22 @@ def _c4_small():
     return prog
 
 
+def test_c4_full_size_bench_configuration(cuda_device):
+    """BASELINE configs[3] at its full size (1280x32x256 fp64) in exactly the launch
+    configuration bench.py times (frozen plan + tuned tiles, perf build), against the
+    full serial oracle (~5 s on the host)."""
+    import sys
+    sys.path.insert(0, os.path.dirname(os.path.dirname(os.path.abspath(__file__))))
+    import bench
+    from _harness import gpu_program
+    prog = bench.load_workload("C4")
+    ref = oracle_outputs(prog, seed=3)
+    p = gpu_program(prog, plan=prog["plans"]["fused"])
+    bench.apply_tuning(p, prog)
+    got = gpu_run(prog, "fused", 3, program=p)
+    assert_close(prog, got, ref)
+
+
 @pytest.mark.parametrize("fmad", [0, 1])
 def test_c4_parity_reduced(cuda_device, fmad):
     """SCALE-LES-shaped 40-kernel DAG (BASELINE configs[3]) on a reduced grid, frozen greedy plan."""

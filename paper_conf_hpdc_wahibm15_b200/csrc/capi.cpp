@@ -207,6 +207,7 @@ sp_status sp_program_set_option(stencil_program *p, const char *key, int64_t v) 
         else if (k == "l2pf") o.l2pf = (int)v;
         else if (k == "pdl") o.pdl = std::max(0, std::min(2, (int)v));
         else if (k == "acc_split") o.acc_split = std::max(1, std::min(4, (int)v));
+        else if (k == "factor") o.factor = v != 0;
         else if (k == "l2_flush") {}
         else fail(SP_E_ARG, "unknown option '" + k + "'");
         if (v < 0 && k != "prefetch") fail(SP_E_ARG, "negative option value");

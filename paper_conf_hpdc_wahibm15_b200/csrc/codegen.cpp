@@ -598,18 +598,52 @@ std::string generate_launch(const stencil_program *p, Launch &L, int index, bool
         // t % ACC) added at the end — independent FMA chains for ILP; the reassociation
         // is within the 1e-12 / 1e-5 tolerance like the FMA contraction itself.
         const int ACC = (p->opt.fmad && G.terms.size() >= 6) ? p->opt.acc_split : 1;
-        auto term_expr = [&](const std::function<std::string(const Src &)> &opd) {
-            std::vector<std::string> part(ACC);
-            for (size_t ti = 0; ti < G.terms.size(); ++ti) {
+        // Perf build, factor=1: the terms sharing one b operand (SCALE-LES-style flux
+        // c_t * a[p+o_t] * m[p]) become m * (sum of c_t * a): one multiply per distinct b
+        // instead of one per term — exact in real arithmetic, a reassociation within the
+        // tolerance like the FMA contraction; the parity build keeps R4's form.
+        std::vector<std::vector<int>> items;  // term indices; >1 entries = one shared b
+        {
+            const bool fac = p->opt.fmad && p->opt.factor;
+            for (int ti = 0; ti < (int)G.terms.size(); ++ti) {
                 const TermR &t = G.terms[ti];
+                bool placed = false;
+                if (fac && t.has_b)
+                    for (auto &it : items) {
+                        const TermR &u = G.terms[it[0]];
+                        if (u.has_b && u.b.stage == t.b.stage && u.b.idx == t.b.idx &&
+                            u.b.dx == t.b.dx && u.b.dy == t.b.dy && u.b.dz == t.b.dz) {
+                            it.push_back(ti);
+                            placed = true;
+                            break;
+                        }
+                    }
+                if (!placed) items.push_back({ti});
+            }
+        }
+        auto term_expr = [&](const std::function<std::string(const Src &)> &opd) {
+            auto scaled = [&](const TermR &t) {
                 std::string a = opd(t.a);
+                if (t.coef == 1.0) return a;
+                if (t.coef == -1.0) return "(-" + a + ")";
+                return (p->opt.coef_const ? coef_ref(t.coef) : "(T)" + lit(t.coef, f32)) + " * " +
+                       a;
+            };
+            std::vector<std::string> part(ACC);
+            for (size_t ii = 0; ii < items.size(); ++ii) {
+                const std::vector<int> &it = items[ii];
                 std::string term;
-                if (t.coef == 1.0) term = a;
-                else if (t.coef == -1.0) term = "(-" + a + ")";
-                else term = (p->opt.coef_const ? coef_ref(t.coef) : "(T)" + lit(t.coef, f32)) +
-                            " * " + a;
-                if (t.has_b) term = "(" + term + ") * " + opd(t.b);
-                std::string &e = part[ti % ACC];
+                if (it.size() == 1) {
+                    const TermR &t = G.terms[it[0]];
+                    term = scaled(t);
+                    if (t.has_b) term = "(" + term + ") * " + opd(t.b);
+                } else {
+                    std::string s;
+                    for (int ti : it) s = s.empty() ? scaled(G.terms[ti]) : "(" + s + ") + " +
+                                                                                scaled(G.terms[ti]);
+                    term = "(" + s + ") * " + opd(G.terms[it[0]].b);
+                }
+                std::string &e = part[ii % ACC];
                 e = e.empty() ? term : "(" + e + ") + " + term;
             }
             std::string e = part[0];

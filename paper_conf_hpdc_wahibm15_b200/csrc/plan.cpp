@@ -275,7 +275,7 @@ static int estimate_regs(const stencil_program *p, const Launch &L) {
 }
 
 // issued instructions per output point (thread-level), for the issue-rate ceiling
-static double estimate_instr(const Launch &L) {
+static double estimate_instr(const Launch &L, bool factor) {
     const double tile = (double)L.tx * L.ty;
     double per_pt = codegen_smem_loads(L) * 1.2, per_step = 60;
     for (const Stage &G : L.st) {
@@ -283,7 +283,17 @@ static double estimate_instr(const Launch &L) {
         double pts = (double)(L.tx + G.ex0 + G.ex1) * (L.ty + G.ey0 + G.ey1);
         double halo = pts - tile;
         int ops = 0;
-        for (const TermR &t : G.terms) ops += 1 + (t.has_b ? 1 : 0);
+        std::vector<const Src *> bs;  // distinct b operands (one multiply each when factored)
+        for (const TermR &t : G.terms) {
+            ops += 1;
+            if (!t.has_b) continue;
+            bool seen = false;
+            for (const Src *b : bs)
+                seen |= b->stage == t.b.stage && b->idx == t.b.idx && b->dx == t.b.dx &&
+                        b->dy == t.b.dy && b->dz == t.b.dz;
+            if (!factor || !seen) ops += 1;
+            bs.push_back(&t.b);
+        }
         per_pt += ops + 1 + (G.stored ? 0.5 : 0) + halo / tile * (2 * ops + 10);
         per_step += 12;
     }
@@ -419,7 +429,7 @@ static void choose_config(const stencil_program *p, Launch &L, bool quick = fals
                                 double t_sm = C.smem_pt * pts / smem_bw;
                                 double t_alu = C.flops_exec * pts / alu;
                                 // issue rate: 4 warp-instructions per SM per cycle at ~70 %
-                                double t_issue = estimate_instr(C) * pts / 32.0 / (sms * 4 * clk * 0.7);
+                                double t_issue = estimate_instr(C, p->opt.fmad && p->opt.factor) * pts / 32.0 / (sms * 4 * clk * 0.7);
                                 // latency hiding by the compute warps (barrier-separated stages)
                                 double warps = std::min<double>(per_sm, std::ceil(ctas / sms)) * nt / 32;
                                 double lat = std::min(1.0, warps / 16.0);

@@ -30,14 +30,15 @@ struct ArrayDesc { std::string name; sp_role role; };
 struct Options {
     int fmad = 1;
     int tile_x = 0, tile_y = 0, zchunk = 0, threads = 0, prefetch = -1;
-    int loader = 0;
+    int loader = 0;  // 0: TMA + mbarrier ring, 1: cooperative ld.global -> st.shared
     int block_x = 0, block_y = 0, block_cby = 0;  // register-block overrides (0 = chooser)
     int zqueue = 0;  // z-queues cost registers/occupancy more than they save (measured r1)
     int suspend_hint = 0;  // ns hint of mbarrier.try_wait (0 = none)
     int l2pf = 0;          // TMA L2 prefetch distance in steps beyond the ring (0 = off)
     int coef_const = 0;    // 1: coefficients in a __constant__ table (r1: 35 % slower)
     int pdl = 1;        // programmatic dependent launch: 1 = fused groups, 2 = all, 0 = off
-    int acc_split = 1;  // >1: interleaved partial sums in the perf build (no gain measured r1)  // 0: TMA + mbarrier ring, 1: cooperative ld.global -> st.shared
+    int acc_split = 1;  // >1: interleaved partial sums in the perf build (no gain measured r1)
+    int factor = 1;     // perf build: terms sharing one b operand are summed, then multiplied once
 };
 
 // ---------------------------------------------------------------- analysis

@@ -116,14 +116,20 @@ int codegen_regs(const stencil_program *p, const Launch &L) {
 }
 
 // shared-memory loads per core point over all statements (z-queue refills count
-// once per step; direct loads once per block position)
+// once per step; direct loads once per block position).  Without z-queues the same
+// (layout, y, x, plane) read by several statements of a step is one load: the
+// generated loads are plain (non-volatile) and ptxas merges them (checked in SASS).
 double codegen_smem_loads(const Launch &L) {
     double loads = 0;
+    std::set<PosKey> all;
     for (const Stage &G : L.st) {
         if (!G.needed) continue;
-        loads += (double)block_positions(L, G).size() / (L.vx * L.vy);
+        auto pos = block_positions(L, G);
+        if (L.zq) loads += (double)pos.size() / (L.vx * L.vy);
+        else
+            for (auto &kv : pos) all.insert(kv.first);
     }
-    return loads;
+    return loads + (double)all.size() / (L.vx * L.vy);
 }
 
 std::string generate_launch(const stencil_program *p, Launch &L, int index, bool fused) {

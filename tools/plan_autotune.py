@@ -178,9 +178,9 @@ def config_candidates(prog):
     tiles = [32, 64] if prog["dtype"] == "f64" else [64, 128]
     out = []
     for tx in tiles:
-        for nt in (128, 256):
+        for nt in (64, 128, 256):
             for bx, by, cb in ((1, 1, 1), (1, 2, 1), (2, 2, 1), (1, 1, 2), (1, 4, 1), (1, 2, 2),
-                               (2, 2, 2), (1, 4, 2)):
+                               (2, 2, 2), (1, 4, 2), (1, 8, 1)):
                 xt = tx // bx
                 if nt % xt or xt > nt or bx * by * cb > 8:
                     continue

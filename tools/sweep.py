@@ -28,6 +28,7 @@ def main():
     ap.add_argument("--grid", action="store_true", help="enumerate tile/block combinations")
     ap.add_argument("--zchunk", type=int, default=32)
     ap.add_argument("--tx", default="32,64")
+    ap.add_argument("--pf", default="", help="comma list of prefetch depths to cross with --grid")
     ap.add_argument("--apply-tuning", action="store_true", help="pin the plan's tuned configs first")
     a = ap.parse_args()
     if a.grid:
@@ -42,9 +43,17 @@ def main():
                             ty = nt // xt * by * cb
                             if ty > 32:
                                 continue
-                            a.cfg.append(f"tile_x={tx},block_x={bx},threads={nt},block_y={by},"
-                                         f"block_cby={cb},tile_y={ty},zchunk={a.zchunk}")
-    prog = bench.load_workload(a.workload)
+                            c = (f"tile_x={tx},block_x={bx},threads={nt},block_y={by},"
+                                 f"block_cby={cb},tile_y={ty},zchunk={a.zchunk}")
+                            if a.pf:
+                                a.cfg += [c + f",prefetch={pf}" for pf in a.pf.split(",")]
+                            else:
+                                a.cfg.append(c)
+    if a.workload.startswith("probe:"):
+        from probe_programs import probe
+        prog = probe(a.workload)
+    else:
+        prog = bench.load_workload(a.workload)
     plan = json.load(open(a.plan))["groups"] if a.plan else bench.plan_of(prog)
     dev = torch.device("cuda:0")
     flush = torch.empty(256 << 20, dtype=torch.uint8, device=dev)

@@ -129,6 +129,7 @@ typedef struct {
     double smem_bytes_pt;     /* shared-memory traffic per point (model)          */
     int32_t block_x, block_y, block_cby; /* per-thread register block of the core  */
     double t_model_us;        /* modelled launch time (tile chooser objective)    */
+    int32_t zqueue;           /* z-reuse policy in effect (the option's values)  */
 } sp_group_report;
 
 typedef struct sp_comm_s sp_comm;
@@ -203,9 +204,14 @@ sp_status fusion_plan_report(const stencil_program *prog, int32_t group, sp_grou
 sp_status sp_plan_source(stencil_program *prog, int32_t mode, char *buf, size_t cap, size_t *len);
 /* Launch configuration (0 = left to the model-driven chooser).  The thread
  * geometry must satisfy tile_x = (tile_x/block_x)*block_x and
- * tile_y = (threads/(tile_x/block_x)) * block_y * block_cby. */
+ * tile_y = (threads/(tile_x/block_x)) * block_y * block_cby.
+ * zqueue selects how values read at several planes are kept across z steps:
+ * 0 = the program's "zqueue" option, 1 = shared-memory loads only, 2 = register
+ * queues per statement, 3 = step-wide register queues of the input columns a
+ * thread owns (results are bit-identical under every policy). */
 typedef struct {
     int32_t tile_x, tile_y, zchunk, threads, prefetch, block_x, block_y, block_cby;
+    int32_t zqueue;
 } sp_tile_config;
 
 /* Empirical tuning hook (the paper's per-kernel block-size tuning, §4.2):

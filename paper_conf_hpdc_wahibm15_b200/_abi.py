@@ -53,7 +53,7 @@ class SpLayout(ctypes.Structure):
 
 class SpTileConfig(ctypes.Structure):
     _fields_ = [(n, ctypes.c_int32) for n in ("tile_x", "tile_y", "zchunk", "threads", "prefetch",
-                                              "block_x", "block_y", "block_cby")]
+                                              "block_x", "block_y", "block_cby", "zqueue")]
 
 
 class SpEdge(ctypes.Structure):
@@ -73,7 +73,8 @@ class SpGroupReport(ctypes.Structure):
                 ("flops_alg", ctypes.c_double), ("bytes_exec", ctypes.c_double),
                 ("flops_exec", ctypes.c_double), ("smem_bytes_pt", ctypes.c_double),
                 ("block_x", ctypes.c_int32), ("block_y", ctypes.c_int32),
-                ("block_cby", ctypes.c_int32), ("t_model_us", ctypes.c_double)]
+                ("block_cby", ctypes.c_int32), ("t_model_us", ctypes.c_double),
+                ("zqueue", ctypes.c_int32)]
 
 
 # every symbol include/stencilfuse.h declares (checked by tests/test_abi.py)

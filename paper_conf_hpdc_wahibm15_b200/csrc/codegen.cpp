@@ -73,6 +73,14 @@ struct PosKey {
 };
 struct PosInfo { int cmin = 1 << 20, cmax = -(1 << 20); };
 
+// z-queue policy: zq 1 = every position read at several planes, per statement;
+// zq 2 = input positions inside the block core only (the column a thread owns),
+// shared by all statements of the step and refilled once per step
+static bool zqueued(const Launch &L, bool stage, int y, int x) {
+    if (L.zq == 1) return true;
+    return L.zq == 2 && !stage && y >= 0 && y < L.vy && x >= 0 && x < L.vx;
+}
+
 static std::map<PosKey, PosInfo> block_positions(const Launch &L, const Stage &G) {
     std::map<PosKey, PosInfo> pos;
     for (const TermR &t : G.terms)
@@ -83,7 +91,8 @@ static std::map<PosKey, PosInfo> block_positions(const Launch &L, const Stage &G
             for (int iy = 0; iy < L.vy; ++iy)
                 for (int jx = 0; jx < L.vx; ++jx) {
                     int c = G.lead + s.dz;
-                    PosInfo &pi = pos[PosKey{s.stage, s.idx, iy + s.dy, jx + s.dx, L.zq ? 0 : c}];
+                    const int y = iy + s.dy, x = jx + s.dx;
+                    PosInfo &pi = pos[PosKey{s.stage, s.idx, y, x, zqueued(L, s.stage, y, x) ? 0 : c}];
                     pi.cmin = std::min(pi.cmin, c);
                     pi.cmax = std::max(pi.cmax, c);
                 }
@@ -125,7 +134,7 @@ double codegen_smem_loads(const Launch &L) {
     for (const Stage &G : L.st) {
         if (!G.needed) continue;
         auto pos = block_positions(L, G);
-        if (L.zq) loads += (double)pos.size() / (L.vx * L.vy);
+        if (L.zq == 1) loads += (double)pos.size() / (L.vx * L.vy);
         else
             for (auto &kv : pos) all.insert(kv.first);
     }
@@ -411,11 +420,30 @@ std::string generate_launch(const stencil_program *p, Launch &L, int index, bool
     auto qname = [&](int m, const PosKey &k) {
         return "zq" + num(m) + "_" + (k.stage ? "S" : "I") + num(k.id) + "_" + sg(k.y) + "_" + sg(k.x);
     };
-    for (size_t m = 0; m < L.st.size(); ++m)
-        for (auto &kv : bpos[m])
-            if (kv.second.cmax > kv.second.cmin)
-                o << "  T " << qname((int)m, kv.first) << "[CBY][" << kv.second.cmax - kv.second.cmin + 1
-                  << "];\n";
+    // zq 2: step-wide input queues (union of the plane ranges of all statements)
+    std::map<PosKey, PosInfo> gq;
+    if (L.zq == 2) {
+        for (size_t m = 0; m < L.st.size(); ++m)
+            for (auto &kv : bpos[m])
+                if (!kv.first.stage && zqueued(L, false, kv.first.y, kv.first.x)) {
+                    PosInfo &g = gq[kv.first];
+                    g.cmin = std::min(g.cmin, kv.second.cmin);
+                    g.cmax = std::max(g.cmax, kv.second.cmax);
+                }
+        for (auto it = gq.begin(); it != gq.end();)
+            it = it->second.cmax > it->second.cmin ? std::next(it) : gq.erase(it);
+    }
+    auto gqname = [&](const PosKey &k) {
+        return "zg_I" + num(k.id) + "_" + sg(k.y) + "_" + sg(k.x);
+    };
+    for (auto &kv : gq)
+        o << "  T " << gqname(kv.first) << "[CBY][" << kv.second.cmax - kv.second.cmin + 1 << "];\n";
+    if (L.zq == 1)
+        for (size_t m = 0; m < L.st.size(); ++m)
+            for (auto &kv : bpos[m])
+                if (kv.second.cmax > kv.second.cmin)
+                    o << "  T " << qname((int)m, kv.first) << "[CBY][" << kv.second.cmax - kv.second.cmin + 1
+                      << "];\n";
     if (!tma) {
         o << "  for (int j = KF; j < min(KF + PF, zc); ++j) {\n";
         batch(o, "    ");
@@ -449,6 +477,9 @@ std::string generate_launch(const stencil_program *p, Launch &L, int index, bool
             for (int c = kv.second.cmin; c <= kv.second.cmax; ++c)
                 basekeys.insert({Lay{kv.first.stage, kv.first.id}, c});
     }
+    for (auto &kv : gq)
+        for (int c = kv.second.cmin; c <= kv.second.cmax; ++c)
+            basekeys.insert({Lay{false, kv.first.id}, c});
     auto bname = [&](const Lay &l, int c) { return "B" + lname(l) + "_" + sg(c); };
     for (auto &bk : basekeys) {
         const Lay &l = bk.first;
@@ -465,6 +496,33 @@ std::string generate_launch(const stencil_program *p, Launch &L, int index, bool
         }
         o << "    T *const " << bname(l, c) << " = " << (l.stage ? "st" : "in") << l.id << " + " << slot
           << " * " << plane << ";\n";
+    }
+    if (!gq.empty()) {
+        auto gaddr = [&](const PosKey &k, int cc) {
+            Lay l{false, k.id};
+            return bname(l, cc) + " + cb_" + lname(l) + " + b * (YT * VY * " + num(lw(l)) + ") + (" +
+                   num(k.y * lw(l) + k.x) + ")";
+        };
+        o << "    #pragma unroll\n    for (int b = 0; b < CBY; ++b) {\n      if (k == KF) {\n";
+        // planes below the input's first loaded plane (statements not yet active at
+        // the first steps) are never consumed: do not touch their (unloaded) slots
+        auto gload = [&](const PosKey &k, int cc) {
+            return "(k + (" + num(cc) + ") >= (" + num(L.in[k.id].qlo) + ") ? *(" + gaddr(k, cc) +
+                   ") : T(0))";
+        };
+        for (auto &kv : gq)
+            for (int cc = kv.second.cmin; cc <= kv.second.cmax; ++cc)
+                o << "        " << gqname(kv.first) << "[b][" << cc - kv.second.cmin << "] = "
+                  << gload(kv.first, cc) << ";\n";
+        o << "      } else {\n";
+        for (auto &kv : gq) {
+            const std::string q = gqname(kv.first);
+            const int r = kv.second.cmax - kv.second.cmin;
+            for (int d = 0; d < r; ++d)
+                o << "        " << q << "[b][" << d << "] = " << q << "[b][" << d + 1 << "];\n";
+            o << "        " << q << "[b][" << r << "] = " << gload(kv.first, kv.second.cmax) << ";\n";
+        }
+        o << "      }\n    }\n";
     }
 
     std::set<int> dirty;
@@ -510,8 +568,9 @@ std::string generate_launch(const stencil_program *p, Launch &L, int index, bool
         };
         // z-queues: advance, refill the newest plane (every step: the pipeline is uniform)
         bool any_q = false;
-        for (auto &kv : pos)
-            if (kv.second.cmax > kv.second.cmin) any_q = true;
+        if (L.zq == 1)
+            for (auto &kv : pos)
+                if (kv.second.cmax > kv.second.cmin) any_q = true;
         if (any_q) {
             o << "      #pragma unroll\n      for (int b = 0; b < CBY; ++b) {\n";
             o << "        if (k == KF) {\n";
@@ -548,7 +607,7 @@ std::string generate_launch(const stencil_program *p, Launch &L, int index, bool
         // direct loads, vectorised along x where aligned
         std::map<std::tuple<bool, int, int, int>, std::set<int>> rows;  // (stage,id,c,y) -> xs
         for (auto &kv : pos)
-            if (kv.second.cmax == kv.second.cmin)
+            if (kv.second.cmax == kv.second.cmin && !gq.count(kv.first))
                 rows[std::make_tuple(kv.first.stage, kv.first.id, kv.second.cmin, kv.first.y)].insert(
                     kv.first.x);
         auto dname = [&](bool st, int id, int cc, int y, int x) {
@@ -594,7 +653,10 @@ std::string generate_launch(const stencil_program *p, Launch &L, int index, bool
                 return "rq" + num(s.idx) + "[b][" + num(iy * VX + jx) + "][" + num(d) + "]";
             }
             int cc = G.lead + s.dz;
-            PosKey k{s.stage, s.idx, iy + s.dy, jx + s.dx, L.zq ? 0 : cc};
+            const int y = iy + s.dy, x = jx + s.dx;
+            PosKey k{s.stage, s.idx, y, x, zqueued(L, s.stage, y, x) ? 0 : cc};
+            auto g = gq.find(k);
+            if (g != gq.end()) return gqname(k) + "[b][" + num(cc - g->second.cmin) + "]";
             const PosInfo &pi = pos.at(k);
             if (pi.cmax > pi.cmin) return qname(m, k) + "[b][" + num(cc - pi.cmin) + "]";
             return dname(s.stage, s.idx, cc, k.y, k.x);

@@ -527,6 +527,7 @@ void analyze_mode(stencil_program *p, bool fused, const std::vector<std::vector<
                 if (c.block_x) p->opt.block_x = c.block_x;
                 if (c.block_y) p->opt.block_y = c.block_y;
                 if (c.block_cby) p->opt.block_cby = c.block_cby;
+                if (c.zqueue) p->opt.zqueue = c.zqueue - 1;
                 try {
                     choose_config(p, L);
                 } catch (...) {
@@ -579,6 +580,7 @@ void fill_report(const stencil_program *p, const Launch &L, sp_group_report *r) 
     r->block_y = L.vy;
     r->block_cby = L.cby;
     r->t_model_us = L.t_model * 1e6;
+    r->zqueue = L.zq;
     (void)p;
 }
 

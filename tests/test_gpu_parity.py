@@ -98,6 +98,23 @@ def test_tile_independence_bitexact(cuda_device, tiles):
         assert_close(prog, got, ref, exact=True)
 
 
+@pytest.mark.parametrize("zqueue", [1, 2])
+def test_zqueue_bitexact(cuda_device, zqueue):
+    """Register z-queues (per statement / step-wide input columns) change no bit (P6)."""
+    cases = [(P.c2(nx=37, ny=19, nz=17), "fused", (TILES[2], TILES[3])),
+             (P.c3(nx=40, ny=21, nz=15), "fission_fused", (TILES[2], TILES[3])),
+             (_c4_small(), "fused", ({}, dict(tile_x=32, tile_y=8, threads=64, block_x=1,
+                                             block_y=4, block_cby=1, zchunk=5)))]
+    for prog, plan, tile_set in cases:
+        ref = oracle_outputs(prog, seed=6)
+        for tiles in tile_set:
+            opts = dict(tiles, fmad=0, zqueue=zqueue)
+            got = gpu_run(prog, "fused", 6, options=opts, plan=prog["plans"][plan])
+            assert_close(prog, got, ref, exact=True)
+        got = gpu_run(prog, "unfused", 6, options={"fmad": 0, "zqueue": zqueue})
+        assert_close(prog, got, ref, exact=True)
+
+
 def test_c2_full_size(cuda_device):
     """BASELINE configs[1] at its full size (256^3 fp64), perf build, vs the oracle."""
     prog = P.c2()

@@ -230,7 +230,8 @@ def tune_configs(prog, groups, tensors, log=print, iters=7):
                 best, bcfg = t, cfg
         if bcfg is not None:
             # refine around the winner: z-chunk, then TMA prefetch distance
-            for key, values in (("zchunk", (16, 64)), ("prefetch", (1, 2, 3))):
+            # and step-wide input z-queues (measured slower on C4's flux groups in r1)
+            for key, values in (("zchunk", (16, 64)), ("prefetch", (1, 2, 3)), ("zqueue", (2,))):
                 base = bcfg
                 for v in values:
                     cfg = dict(base, **{key: v})

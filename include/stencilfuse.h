@@ -159,8 +159,19 @@ sp_status stencil_program_layout(const stencil_program *prog, sp_layout *out);
 sp_status stencil_program_bind(stencil_program *prog, int32_t array, void *dev_ptr);
 
 /* Tuning/parity options; must precede fusion_plan_set / the first run.
+ * Unknown keys or negative values: SP_E_ARG.  Results are bit-identical under
+ * every option except "fmad"/"factor" (which select the perf build, R4/R17).
  *   "fmad"      0|1  FMA contraction in generated code (default 1; 0 = parity build)
+ *   "factor"    0|1  perf build: terms sharing one multiplier summed first (default 1)
  *   "tile_x", "tile_y", "zchunk", "threads", "prefetch"   override the tile chooser
+ *   "block_x", "block_y", "block_cby"   register block of a thread (0 = chooser)
+ *   "zqueue"    0..2  z-reuse policy (see sp_tile_config.zqueue)
+ *   "loader"    0 = TMA + mbarrier ring (default), 1 = cooperative loads
+ *   "pdl"       0|1|2 programmatic dependent launch: off / fused groups / all
+ *   "zwave"     S > 0: fused mode runs the z-wave schedule (sp_plan_wave_offsets)
+ *   "zwave_streams" 1..8 waves in flight for "zwave" (default 2)
+ *   "suspend_hint", "coef_const", "l2pf", "acc_split"   measured-off experiments
+ *   "num_sms"   SM count assumed by the tile chooser (default 148)
  *   "l2_flush"  unused by the library (reserved) */
 sp_status sp_program_set_option(stencil_program *prog, const char *key, int64_t value);
 
@@ -227,6 +238,16 @@ sp_status sp_plan_tune(stencil_program *prog, int32_t mode, int32_t launch, cons
  * exactly this exchange before the launch's boundary chunks. */
 sp_status sp_plan_exchange(stencil_program *prog, int32_t mode, int32_t launch, int32_t cap,
                            int32_t *arrays, int32_t *n, int32_t *depth);
+/* z-wave schedule of the fused mode (options "zwave" = S planes per wave,
+ * "zwave_streams" = waves in flight on that many streams; single rank only).
+ * In wave w, launch i evaluates output planes [w*S - off_i, (w+1)*S - off_i)
+ * of the slab; the skew off_i >= 0 is the smallest that keeps every plane a
+ * launch reads or writes disjoint from the planes of concurrently running or
+ * later-issued waves of other launches (RAW: off_i >= off_j + z-reach above,
+ * WAR: off_i >= off_j + z-reach below, WAW: off_i >= off_j for j < i), so
+ * results are bit-identical to plan order.  Writes up to cap offsets, *n = the
+ * number of fused launches.  Host-only (no GPU needed). */
+sp_status sp_plan_wave_offsets(stencil_program *prog, int32_t cap, int32_t *off, int32_t *n);
 /* JIT-compile (NVRTC, sm_100a) without launching; needs no GPU. */
 sp_status sp_compile(stencil_program *prog, int32_t mode);
 

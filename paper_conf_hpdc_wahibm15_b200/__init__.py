@@ -279,6 +279,14 @@ class Program:
                                       ctypes.byref(n), ctypes.byref(depth)))
         return [self.names[buf[j]] for j in range(n.value)], depth.value
 
+    def wave_offsets(self):
+        """Plane skew of each fused launch in the z-wave schedule (option "zwave")."""
+        n = ctypes.c_int32()
+        _check(lib().sp_plan_wave_offsets(self.handle, 0, None, ctypes.byref(n)))
+        buf = (ctypes.c_int32 * max(1, n.value))()
+        _check(lib().sp_plan_wave_offsets(self.handle, n.value, buf, ctypes.byref(n)))
+        return [buf[j] for j in range(n.value)]
+
     def compile(self, mode):
         _check(lib().sp_compile(self.handle, self._mode(mode)))
 

@@ -83,7 +83,7 @@ EXPORTS = [
     "stencil_program_destroy", "stencil_program_layout", "stencil_program_bind",
     "sp_program_set_option", "sp_program_counts", "sp_program_edges", "sp_fission_components",
     "fusion_plan_set", "sp_plan_greedy", "sp_plan_count", "sp_plan_report", "fusion_plan_report", "sp_plan_source",
-    "sp_plan_exchange", "sp_plan_tune", "sp_compile", "run_unfused", "run_fused", "sp_run_launch", "exchange_halos", "sp_last_error",
+    "sp_plan_exchange", "sp_plan_wave_offsets", "sp_plan_tune", "sp_compile", "run_unfused", "run_fused", "sp_run_launch", "exchange_halos", "sp_last_error",
 ]
 
 _lib = None
@@ -116,6 +116,7 @@ def lib():
             "sp_plan_source": [vp, i32, ctypes.c_char_p, ctypes.c_size_t, P(ctypes.c_size_t)],
             "sp_compile": [vp, i32],
             "sp_plan_exchange": [vp, i32, i32, i32, P(i32), P(i32), P(i32)],
+            "sp_plan_wave_offsets": [vp, i32, P(i32), P(i32)],
             "sp_plan_tune": [vp, i32, i32, P(SpTileConfig)],
             "run_unfused": [vp, vp],
             "run_fused": [vp, vp],

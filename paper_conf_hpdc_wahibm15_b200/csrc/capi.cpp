@@ -85,10 +85,118 @@ static int exchange_set(const Launch &L, std::vector<int> &arrays) {
     return std::max(L.z_below, L.z_above);
 }
 
+// ---------------------------------------------------------------- z-wave schedule
+// The step is cut into waves of S planes; in wave w launch i covers planes
+// [w*S - off_i, (w+1)*S - off_i).  The skew off_i makes every wave of a launch
+// independent of later waves of earlier launches:
+//   RAW  (j < i stores X, i reads X up to ahi planes above its chunk):  off_i >= off_j + ahi
+//   WAR  (j < i, j reads X down to qlo planes below its chunk, i stores X): off_i >= off_j - qlo
+//   WAW  (j < i both store X): off_i >= off_j
+// so the result is the plan's result (bit-exact: every point is evaluated by the
+// same code, only the chunking changes, P6).  Consecutive launches of one wave
+// touch the same few-MB z-slab, so a producer's output is still in the 126 MB L2
+// when its consumer reads it (cross-group locality the paper gets from fusion).
+static void wave_offsets(const stencil_program *p, Mode &m) {
+    const size_t n = m.launches.size();
+    m.wave_off.assign(n, 0);
+    std::vector<std::vector<int>> stores(n);
+    for (size_t i = 0; i < n; ++i)
+        for (const Stage &G : m.launches[i].st)
+            if (G.stored) stores[i].push_back(G.out);
+    auto stores_arr = [&](size_t i, int a) {
+        return std::find(stores[i].begin(), stores[i].end(), a) != stores[i].end();
+    };
+    for (size_t i = 0; i < n; ++i) {
+        if (m.launches[i].dead) continue;
+        int off = 0;
+        for (size_t j = 0; j < i; ++j) {
+            if (m.launches[j].dead) continue;
+            for (const Input &I : m.launches[i].in)
+                if (stores_arr(j, I.arr)) off = std::max(off, m.wave_off[j] + std::max(0, I.ahi));
+            for (const Input &I : m.launches[j].in)
+                if (stores_arr(i, I.arr)) off = std::max(off, m.wave_off[j] + std::max(0, -I.qlo));
+            for (int a : stores[i])
+                if (stores_arr(j, a)) off = std::max(off, m.wave_off[j]);
+        }
+        m.wave_off[i] = off;
+    }
+    (void)p;
+}
+
+static void run_waves(stencil_program *p, Mode &m, void *stream) {
+    if (m.wave_off.size() != m.launches.size()) wave_offsets(p, m);
+    const int S = p->opt.zwave, ns = std::max(1, p->opt.zwave_streams);
+    const int nz = (int)p->grid.nz_local, n = (int)m.launches.size();
+    int maxoff = 0;
+    for (int o : m.wave_off) maxoff = std::max(maxoff, o);
+    const int nw = (nz + maxoff + S - 1) / S;
+    auto range = [&](int w, int i, int *z0, int *z1) {
+        *z0 = std::max(0, w * S - m.wave_off[i]);
+        *z1 = std::min(nz, (w + 1) * S - m.wave_off[i]);
+        return *z1 > *z0;
+    };
+    auto go = [&](int w, int i, void *s) {
+        int z0, z1;
+        if (m.launches[i].dead || !range(w, i, &z0, &z1)) return false;
+        const int zc = m.launches[i].zc;
+        launch(p, m, i, s, 0, 1, (z1 - z0 + zc - 1) / zc, z0, z1);
+        return true;
+    };
+    if (ns == 1) {
+        for (int w = 0; w < nw; ++w)
+            for (int i = 0; i < n; ++i) go(w, i, stream);
+        return;
+    }
+    // ns streams, wave w on stream w % ns; (w, i) waits on (w-1, i) (and, by stream
+    // order, on (w, j < i)): the skew keeps everything else that may run
+    // concurrently (waves w-1.. of later launches) on disjoint planes
+    while ((int)p->wave_streams.size() < ns) {
+        cudaStream_t s;
+        if (cudaStreamCreateWithFlags(&s, cudaStreamNonBlocking) != cudaSuccess)
+            fail(SP_E_CUDA, "cudaStreamCreate");
+        p->wave_streams.push_back(s);
+    }
+    const size_t nev = (size_t)ns * n + 1 + ns;
+    while (p->wave_events.size() < nev) {
+        cudaEvent_t ev;
+        if (cudaEventCreateWithFlags(&ev, cudaEventDisableTiming) != cudaSuccess)
+            fail(SP_E_CUDA, "cudaEventCreate");
+        p->wave_events.push_back(ev);
+    }
+    auto ev = [&](size_t k) { return (cudaEvent_t)p->wave_events[k]; };
+    auto st = [&](int k) { return (cudaStream_t)p->wave_streams[k]; };
+    const size_t fork = (size_t)ns * n, join0 = fork + 1;
+    if (cudaEventRecord(ev(fork), (cudaStream_t)stream) != cudaSuccess)
+        fail(SP_E_CUDA, "event record");
+    for (int k = 0; k < ns; ++k)
+        if (cudaStreamWaitEvent(st(k), ev(fork), 0) != cudaSuccess) fail(SP_E_CUDA, "stream wait");
+    std::vector<char> prev(n, 0), cur(n, 0);
+    for (int w = 0; w < nw; ++w) {
+        cudaStream_t s = st(w % ns);
+        for (int i = 0; i < n; ++i) {
+            if (prev[i] && cudaStreamWaitEvent(s, ev((size_t)((w - 1) % ns) * n + i), 0) != cudaSuccess)
+                fail(SP_E_CUDA, "stream wait");
+            cur[i] = go(w, i, s);
+            if (cur[i] && cudaEventRecord(ev((size_t)(w % ns) * n + i), s) != cudaSuccess)
+                fail(SP_E_CUDA, "event record");
+        }
+        prev.swap(cur);
+    }
+    for (int k = 0; k < ns; ++k) {
+        if (cudaEventRecord(ev(join0 + k), st(k)) != cudaSuccess ||
+            cudaStreamWaitEvent((cudaStream_t)stream, ev(join0 + k), 0) != cudaSuccess)
+            fail(SP_E_CUDA, "event record/wait");
+    }
+}
+
 static void run_mode(stencil_program *p, int mode, void *stream) {
     Mode &m = mode_of(p, mode);
     load_mode(p, m);
     const bool multi = p->comm && p->comm->nranks > 1;
+    if (mode == 1 && p->opt.zwave > 0 && !multi) {
+        run_waves(p, m, stream);
+        return;
+    }
     for (size_t i = 0; i < m.launches.size(); ++i) {
         Launch &L = m.launches[i];
         if (L.dead) continue;
@@ -162,6 +270,8 @@ void stencil_program_destroy(stencil_program *p) {
         unload_mode(p->unfused);
         unload_mode(p->fused);
         for (void *e : p->events) cudaEventDestroy((cudaEvent_t)e);
+        for (void *e : p->wave_events) cudaEventDestroy((cudaEvent_t)e);
+        for (void *s : p->wave_streams) cudaStreamDestroy((cudaStream_t)s);
     });
     delete p;
 }
@@ -208,6 +318,8 @@ sp_status sp_program_set_option(stencil_program *p, const char *key, int64_t v) 
         else if (k == "pdl") o.pdl = std::max(0, std::min(2, (int)v));
         else if (k == "acc_split") o.acc_split = std::max(1, std::min(4, (int)v));
         else if (k == "factor") o.factor = v != 0;
+        else if (k == "zwave") o.zwave = (int)v;
+        else if (k == "zwave_streams") o.zwave_streams = std::max(1, std::min(8, (int)v));
         else if (k == "l2_flush") {}
         else fail(SP_E_ARG, "unknown option '" + k + "'");
         if (v < 0 && k != "prefetch") fail(SP_E_ARG, "negative option value");
@@ -354,6 +466,16 @@ sp_status sp_plan_exchange(stencil_program *p, int32_t mode, int32_t launch, int
         *depth = m.launches[launch].dead ? 0 : exchange_set(m.launches[launch], a);
         *n = (int)a.size();
         for (int i = 0; i < std::min<int>(cap, (int)a.size()); ++i) arrays[i] = a[i];
+    });
+}
+
+sp_status sp_plan_wave_offsets(stencil_program *p, int32_t cap, int32_t *off, int32_t *n) {
+    return guard([&] {
+        if (!p || !n || (cap > 0 && !off)) fail(SP_E_ARG, "null argument");
+        Mode &m = mode_of(p, 1);
+        wave_offsets(p, m);
+        *n = (int)m.wave_off.size();
+        for (int i = 0; i < std::min<int>(cap, *n); ++i) off[i] = m.wave_off[i];
     });
 }
 

@@ -256,13 +256,14 @@ static void build_params(stencil_program *p, Mode &m) {
 }
 
 void launch(stencil_program *p, Mode &m, int i, void *stream, int chunk_first, int chunk_step,
-            int nchunks) {
+            int nchunks, int z_base, int z_end) {
     Launch &L = m.launches[i];
     if (L.dead || nchunks <= 0) return;
     build_params(p, m);
     unsigned char *base = m.params[i][0].b;
-    int32_t ints[2] = {chunk_first, chunk_step};
-    std::memcpy(base + L.int_off, ints, 8);
+    if (z_end < 0) z_end = (int)p->grid.nz_local;
+    int32_t ints[4] = {chunk_first, chunk_step, z_base, z_end};
+    std::memcpy(base + L.int_off, ints, 16);
     void *args[] = {base};
     if (L.pdl) {
         // programmatic dependent launch: the kernel's prologue may overlap the previous

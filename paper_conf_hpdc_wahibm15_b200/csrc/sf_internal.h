@@ -39,6 +39,8 @@ struct Options {
     int pdl = 1;        // programmatic dependent launch: 1 = fused groups, 2 = all, 0 = off
     int acc_split = 1;  // >1: interleaved partial sums in the perf build (no gain measured r1)
     int factor = 1;     // perf build: terms sharing one b operand are summed, then multiplied once
+    int zwave = 0;          // z-wave schedule: planes per wave (0 = one launch per group per step)
+    int zwave_streams = 2;  // waves in flight (streams) of the z-wave schedule
 };
 
 // ---------------------------------------------------------------- analysis
@@ -126,6 +128,7 @@ struct Mode {
     uint64_t maps_version = ~0ull;
     struct alignas(64) Blk { unsigned char b[64]; };
     std::vector<std::vector<Blk>> params;  // per launch: tensor maps + pointers + ints
+    std::vector<int> wave_off;  // z-wave schedule: plane offset (skew) per launch
 };
 
 }  // namespace sf
@@ -155,6 +158,7 @@ struct stencil_program_s {
     std::vector<std::vector<int>> plan_groups;  // gids per group
     int num_sms = 148;
     std::vector<void *> events;  // cudaEvent_t pool for exchange overlap
+    std::vector<void *> wave_streams, wave_events;  // z-wave schedule: streams, events
     std::map<int, sp_tile_config> tune_fused, tune_unfused;  // sp_plan_tune overrides
 };
 
@@ -183,8 +187,10 @@ double codegen_smem_loads(const Launch &L);  // shared-memory loads per core poi
 // jit.cpp
 void compile_mode(stencil_program *p, Mode &m);
 void load_mode(stencil_program *p, Mode &m);
+// chunks chunk_first + c*chunk_step (c < nchunks) of the z range [z_base, z_end)
+// (z_end < 0: the whole local slab); chunk c starts at plane z_base + chunk*zc
 void launch(stencil_program *p, Mode &m, int i, void *stream, int chunk_first, int chunk_step,
-            int nchunks);
+            int nchunks, int z_base = 0, int z_end = -1);
 void ensure_cuda();
 void unload_mode(Mode &m);
 

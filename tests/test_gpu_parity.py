@@ -157,3 +157,43 @@ def test_c4_parity_reduced(cuda_device, fmad):
     for mode in ("unfused", "fused"):
         got = gpu_run(prog, mode, 7, options={"fmad": fmad}, plan=prog["plans"]["fused"])
         assert_close(prog, got, ref, exact=(fmad == 0))
+
+
+WAVES = [(1, 1), (3, 2), (5, 4), (8, 3), (16, 2)]
+
+
+@pytest.mark.parametrize("zwave,streams", WAVES, ids=[f"S{a}x{b}" for a, b in WAVES])
+def test_zwave_schedule_bitexact(cuda_device, zwave, streams):
+    """z-wave schedule (launch i runs planes [wS - off_i, (w+1)S - off_i) per wave,
+    waves in flight on several streams): bit-exact with the oracle (P6) for plans with
+    RAW, WAR and WAW dependencies between groups, incl. tiny waves (S=1) that put
+    every hazard distance at its minimum."""
+    cases = [(P.c2(nx=37, ny=19, nz=17), ["fused"]),
+             (P.c3(nx=40, ny=21, nz=23), ["fused", "fission_fused"]),
+             (P.c5(nx=40, ny=23, nz=19), ["fused"]),
+             (P.resize(P.chain3(), 33, 17, 13), ["fused"]),
+             (_c4_small(), ["fused"])]
+    for prog, plans in cases:
+        ref = oracle_outputs(prog, seed=8)
+        for plan in plans:
+            opts = {"fmad": 0, "zwave": zwave, "zwave_streams": streams, "zchunk": 4}
+            got = gpu_run(prog, "fused", 8, options=opts, plan=prog["plans"][plan], repeat=2)
+            assert_close(prog, got, ref, exact=True)
+
+
+def test_zwave_full_size_c4(cuda_device):
+    """The bench's C4 launch configuration under the z-wave schedule, perf build, vs the
+    plain plan order bit-exactly (same kernels, only the z-chunking differs)."""
+    import sys
+    sys.path.insert(0, os.path.dirname(os.path.dirname(os.path.abspath(__file__))))
+    import bench
+    from _harness import gpu_program
+    prog = bench.load_workload("C4")
+    outs = {}
+    for zw in (0, 32):
+        p = gpu_program(prog, options={"zwave": zw, "zwave_streams": 3},
+                        plan=prog["plans"]["fused"])
+        bench.apply_tuning(p, prog)
+        outs[zw] = gpu_run(prog, "fused", 9, program=p, repeat=2)
+    for n in outs[0]:
+        assert outs[0][n].tobytes() == outs[32][n].tobytes(), n

@@ -300,3 +300,31 @@ def test_greedy_plan_is_legal_and_reduces_traffic():
     assert fused < 0.7 * unfused
     refs = [r for g in plan for r in g]
     assert len(refs) == len(set(refs)) == sum(len(k["stmts"]) for k in prog["kernels"])
+
+
+def test_wave_offsets_raw_reach():
+    """z-wave skew: K3 reads T2 one plane above (dz=+1), so it trails K2 by one plane;
+    point-wise and in-plane reads need no skew."""
+    prog = P.resize(P.chain3(), 16, 8, 12)
+    p = Program(prog)
+    p.set_plan([["K1"], ["K2"], ["K3"]])
+    assert p.wave_offsets() == [0, 0, 1]
+    p.set_plan(prog["plans"]["fused"])
+    assert p.wave_offsets() == [0]
+
+
+def test_wave_offsets_war_waw():
+    """WAR: K2 overwrites X, which K1 reads two planes below, so K2 trails K1 by 2;
+    K3 reads K2's X point-wise (RAW, no reach) and inherits the skew."""
+    T = P.tap
+    prog = {"name": "war", "dtype": "f64", "grid": {"nx": 16, "ny": 8, "nz": 12, "ghost": [1, 1, 2]},
+            "arrays": [{"name": n, "role": r} for n, r in
+                       (("A", "in"), ("B", "in"), ("X", "temp"), ("Y", "temp"), ("O", "out"))],
+            "kernels": [P.kernel("K0", P.stmt("X", [{"c": 1.0, "a": T("A", (0, 0, 0))}])),
+                        P.kernel("K1", P.stmt("Y", [{"c": 1.0, "a": T("X", (0, 0, -2))}])),
+                        P.kernel("K2", P.stmt("X", [{"c": 1.0, "a": T("B", (0, 0, 0))}])),
+                        P.kernel("K3", P.stmt("O", [{"c": 1.0, "a": T("Y", (0, 0, 0))},
+                                                    {"c": 1.0, "a": T("X", (0, 0, 0))}]))]}
+    p = Program(prog)
+    p.set_plan([["K0"], ["K1"], ["K2"], ["K3"]])
+    assert p.wave_offsets() == [0, 0, 2, 2]

@@ -1,5 +1,4 @@
 export PYTHONUNBUFFERED=1
-timeout 300 python tools/step_series.py C4 --steps 600 --window 20 > gpurun_out/ser31.log 2>&1
-timeout 300 python tools/step_series.py C4 --steps 400 --window 20 --mode unfused > gpurun_out/ser31u.log 2>&1
-nvidia-smi -q -d POWER,CLOCK,PERFORMANCE > gpurun_out/smi31.txt 2>&1
-head -2 gpurun_out/ser31.log; head -2 gpurun_out/ser31u.log
+timeout 700 python tools/sweep.py C4 --group 2 --grid --tx 32,64,128,256 --zchunk 32 --pf 1,2,3 > gpurun_out/sw2_g2.log 2>&1
+timeout 700 python tools/sweep.py C4 --group 5 --grid --tx 32,64,128 --zchunk 32 --pf 2,3 > gpurun_out/sw2_g5.log 2>&1
+tail -3 gpurun_out/sw2_g2.log

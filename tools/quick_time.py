@@ -38,7 +38,7 @@ def main():
         v = field_torch(1, aid, p.n, p.ghost, prog["dtype"], dev)
         p.padded_view(p.tensors[arr["name"]]).copy_(v)
     pts = p.n[0] * p.n[1] * p.n[2]
-    flush = torch.empty(256 << 20, dtype=torch.uint8, device=dev)
+    flush = torch.ones(32 << 20, dtype=torch.float64, device=dev)  # read-only L2 flush (no dirty lines)
     plans = a.plans or [k for k in prog["plans"] if k != "unfused"]
     for mode, plan in [("unfused", None)] + [("fused", pl) for pl in plans]:
         if plan:
@@ -52,7 +52,7 @@ def main():
         for i, r in enumerate(reps):
             ts = []
             for _ in range(a.iters):
-                flush.zero_()
+                flush.sum()
                 s, e = torch.cuda.Event(True), torch.cuda.Event(True)
                 s.record()
                 p.run_launch(mode, i)

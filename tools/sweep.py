@@ -56,7 +56,7 @@ def main():
         prog = bench.load_workload(a.workload)
     plan = json.load(open(a.plan))["groups"] if a.plan else bench.plan_of(prog)
     dev = torch.device("cuda:0")
-    flush = torch.empty(256 << 20, dtype=torch.uint8, device=dev)
+    flush = torch.ones(32 << 20, dtype=torch.float64, device=dev)  # read-only L2 flush (no dirty lines)
     base = None
     pts = prog["grid"]["nx"] * prog["grid"]["ny"] * prog["grid"]["nz"]
     for cfg in [""] + a.cfg:
@@ -82,7 +82,7 @@ def main():
             torch.cuda.synchronize()
             ts = []
             for _ in range(a.iters):
-                flush.zero_()
+                flush.sum()
                 s, e = torch.cuda.Event(True), torch.cuda.Event(True)
                 s.record()
                 p.run_launch(a.mode, a.group)

@@ -58,9 +58,9 @@ def apply_tuning(p, prog):
                 p.tune("fused", i, c)
 
 
-def plan_of(prog):
-    if "fused" in prog["plans"]:
-        return prog["plans"]["fused"]
+def plan_of(prog, name="fused"):
+    if name in prog["plans"]:
+        return prog["plans"][name]
     from paper_conf_hpdc_wahibm15_b200 import Program
     return Program(prog).plan_greedy()
 
@@ -151,7 +151,7 @@ def run_ours(args):
     dev = torch.device("cuda", local if world > 1 else 0)
     torch.cuda.set_device(dev)
     prog = load_workload(args.workload)
-    plan = plan_of(prog)
+    plan = plan_of(prog, args.plan)
     nz = prog["grid"]["nz"]
     # deep halo needed by the plan's accumulated z-reach (probe on the local grid)
     probe = Program(prog)
@@ -320,7 +320,8 @@ def run_ours(args):
             "dtype": prog["dtype"], "data": "synthetic: seeded splitmix64 uniform[-1,1) fields",
             "config": {"workload": args.workload, "grid_per_gpu": [prog["grid"]["nx"], prog["grid"]["ny"], nz],
                        "kernels": n_kernels, "arrays": len(prog["arrays"]),
-                       "fused_groups": len(live_f), "parallelism": f"z-slab x{world}",
+                       "plan": args.plan, "fused_groups": len(live_f),
+                       "parallelism": f"z-slab x{world}",
                        "l2": "no flush: per-GPU working set > 126 MB L2"},
             "hbm_gbs_alg": alg_step / (step_ms * 1e-3) / 1e9,
             "roofline_step": {"achieved": alg_step / (step_ms * 1e-3) / 1e9, "peak": peak,
@@ -415,6 +416,7 @@ def main():
     ap.add_argument("--warmup", type=int, default=10)
     ap.add_argument("--workload", default="C4", choices=["C1", "C2", "C3", "C4", "C5"])
     ap.add_argument("--impl", default="ours", choices=["ours", "reference"])
+    ap.add_argument("--plan", default="fused", help="named plan of the workload (e.g. C3 fission_fused)")
     ap.add_argument("--no-cpu", action="store_true", help="skip the cpu_baseline leg")
     args = ap.parse_args()
     if args.warmup < 3:

@@ -73,8 +73,20 @@ typedef struct { double coef; sp_tap a; int32_t has_b; sp_tap b; } sp_term;
 typedef struct { int32_t out; int32_t n_terms; const sp_term *terms; } sp_stmt;
 
 /* A kernel: ordered statements executed per point (reading R3:
- * an array written by the kernel may be read by it only at offset 0). */
-typedef struct { const char *name; int32_t n_stmts; const sp_stmt *stmts; } sp_kernel;
+ * an array written by the kernel may be read by it only at offset 0).
+ * box: the kernel's loop bounds (§5.5.2, kernels with "shorter loops",
+ * e.g. boundary kernels on one plane): NULL = the whole interior,
+ * else 6 values {x0, x1, y0, y1, z0, z1}, half-open, in GLOBAL interior
+ * coordinates, 0 <= x0 <= x1 <= nx, 0 <= y0 <= y1 <= ny, 0 <= z0 <= z1 <=
+ * nz_global (copied at create time).  The kernel's statements write exactly
+ * the interior points inside the box; every other point of their output
+ * arrays keeps its stored value (reading R2').  SP_E_PROGRAM if out of range. */
+typedef struct {
+    const char *name;
+    int32_t n_stmts;
+    const sp_stmt *stmts;
+    const int64_t *box;
+} sp_kernel;
 
 typedef struct { const char *name; sp_role role; } sp_array_desc;
 
@@ -130,6 +142,10 @@ typedef struct {
     int32_t block_x, block_y, block_cby; /* per-thread register block of the core  */
     double t_model_us;        /* modelled launch time (tile chooser objective)    */
     int32_t zqueue;           /* z-reuse policy in effect (the option's values)  */
+    int32_t est_regs;         /* registers per thread the chooser assumed        */
+    int32_t warmup_steps;     /* z steps a chunk runs before its first plane      */
+    int32_t prefetch;         /* TMA batches in flight ahead of the compute warps */
+    double instr_pt;          /* modelled issued instructions per point (thread)  */
 } sp_group_report;
 
 typedef struct sp_comm_s sp_comm;

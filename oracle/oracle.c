@@ -8,6 +8,7 @@
  *                                                     statement-wise = kernel-wise
  *                                                     under reading R3)
  *     for k, j, i over the interior (∩ box)          (R1, R2)
+ *                 ∩ the statement's loop bounds      (R2': kernels with shorter loops)
  *       acc = T(S.term[0]); acc = acc + T(S.term[t]) (R4: fixed left-to-right order)
  *       S.out[i,j,k] = acc
  *
@@ -77,9 +78,16 @@ static void clip_box(const or_grid *g, const long *box, long r[6]) {
         for (int s = 0; s < n_stmts; ++s) {                                            \
             const or_stmt *S = &stmts[s];                                              \
             STORE *out = arrays[S->out];                                               \
-            for (long k = r[4]; k < r[5]; ++k)                                         \
-                for (long j = r[2]; j < r[3]; ++j)                                     \
-                    for (long i = r[0]; i < r[1]; ++i) {                               \
+            long q[6]; /* points evaluated: interior, box, statement loop bounds */    \
+            for (int d = 0; d < 6; ++d) q[d] = r[d];                                   \
+            if (S->has_box)                                                            \
+                for (int d = 0; d < 3; ++d) {                                          \
+                    if (S->box[2 * d] > q[2 * d]) q[2 * d] = S->box[2 * d];            \
+                    if (S->box[2 * d + 1] < q[2 * d + 1]) q[2 * d + 1] = S->box[2 * d + 1]; \
+                }                                                                      \
+            for (long k = q[4]; k < q[5]; ++k)                                         \
+                for (long j = q[2]; j < q[3]; ++j)                                     \
+                    for (long i = q[0]; i < q[1]; ++i) {                               \
                         long p = L.base + k * L.sz + j * L.sy + i * L.sx;              \
                         REAL acc = 0;                                                  \
                         for (int t = 0; t < S->n_terms; ++t) {                         \

@@ -11,7 +11,8 @@
  *   single run" (§6.1.2).  The oracle is therefore the ORIGINAL program:
  *   every kernel, in host invocation order (the OEG total order, §3.2.3),
  *   every statement of the kernel in order (reading R3 in DESIGN.md), every
- *   interior point of the grid (R1/R2), accumulating the statement's terms left
+ *   interior point of the grid inside the kernel's loop bounds (R1/R2/R2'),
+ *   accumulating the statement's terms left
  *   to right (R4):
  *       acc = T(term0);  acc = acc + T(term_t) for t = 1..;   out[p] = acc
  *       T(term) = coef * a[p+oa]            or   (coef * a[p+oa]) * b[p+ob]
@@ -40,7 +41,10 @@ extern "C" {
 
 typedef struct { int arr, dx, dy, dz; } or_tap;
 typedef struct { double coef; or_tap a; int has_b; or_tap b; } or_term;
-typedef struct { int out; int n_terms; const or_term *terms; } or_stmt;
+/* has_box: the statement's kernel iterates only box = [i0,i1) x [j0,j1) x [k0,k1)
+ * of the interior (its loop bounds, §5.5.2 "shorter loops";
+ * reading R2' in DESIGN.md): points outside it are not written. */
+typedef struct { int out; int n_terms; const or_term *terms; int has_box; long box[6]; } or_stmt;
 typedef struct { long nx, ny, nz; int hx, hy, hz; } or_grid;
 
 /* Runs n_stmts statements (kernels flattened in program order) over the grid.

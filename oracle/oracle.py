@@ -35,7 +35,8 @@ class OrTerm(ctypes.Structure):
 
 class OrStmt(ctypes.Structure):
     _fields_ = [("out", ctypes.c_int), ("n_terms", ctypes.c_int),
-                ("terms", ctypes.POINTER(OrTerm))]
+                ("terms", ctypes.POINTER(OrTerm)), ("has_box", ctypes.c_int),
+                ("box", ctypes.c_long * 6)]
 
 
 class OrGrid(ctypes.Structure):
@@ -91,6 +92,8 @@ class OracleProgram:
         self.roles = {a["name"]: a["role"] for a in prog["arrays"]}
         self._validate()
         stmts = [s for k in prog["kernels"] for s in k["stmts"]]
+        # loop bounds (reading R2'): the kernel's box, in global interior coordinates
+        self.boxes = [k.get("box") for k in prog["kernels"] for _ in k["stmts"]]
         self._keep = []
         self.c_stmts = (OrStmt * len(stmts))()
         for si, s in enumerate(stmts):
@@ -106,6 +109,16 @@ class OracleProgram:
             self.c_stmts[si].n_terms = len(s["terms"])
             self.c_stmts[si].terms = terms
         self.n_stmts = len(stmts)
+        self._set_origin((0, 0, 0))
+
+    def _set_origin(self, origin):
+        """Statement boxes in the coordinates of a window whose interior point
+        (0,0,0) is the global point `origin`."""
+        for si, b in enumerate(self.boxes):
+            self.c_stmts[si].has_box = int(b is not None)
+            if b is not None:
+                for d in range(6):
+                    self.c_stmts[si].box[d] = int(b[d]) - int(origin[d // 2])
 
     def _tap(self, t):
         return OrTap(self.index[t[0]], int(t[1]), int(t[2]), int(t[3]))
@@ -145,14 +158,16 @@ class OracleProgram:
             ptrs[i] = a.ctypes.data_as(ctypes.POINTER(real))
         return ptrs
 
-    def run(self, arrays: dict, box=None, wide=False, n=None):
+    def run(self, arrays: dict, box=None, wide=False, n=None, origin=(0, 0, 0)):
         """Evaluate in place on dense padded arrays {name: ndarray}.
 
         box: optional (i0,i1,j0,j1,k0,k1) restricting the evaluated points;
         wide: fp32 programs only — evaluate in binary64 (error bound check);
-        n: interior size of the arrays if they are a window, not the program grid.
+        n: interior size of the arrays if they are a window, not the program grid;
+        origin: global coordinates of the window's interior point (0,0,0).
         """
         lib = load_library()
+        self._set_origin(origin)
         grid = self._grid(n)
         real = ctypes.c_double if self.dtype == "f64" else ctypes.c_float
         ptrs = self._ptrs(arrays, real)

@@ -128,6 +128,10 @@ class Program:
             kernels[ki].name = nm
             kernels[ki].n_stmts = len(k["stmts"])
             kernels[ki].stmts = stmts
+            if k.get("box") is not None:
+                box = (ctypes.c_int64 * 6)(*[int(v) for v in k["box"]])
+                self._keep.append(box)
+                kernels[ki].box = box
         self.comm = comm
         self.handle = ctypes.c_void_p()
         _check(lib().stencil_program_create(ctypes.byref(grid), len(self.names), arrays,

@@ -27,7 +27,7 @@ class SpStmt(ctypes.Structure):
 
 class SpKernel(ctypes.Structure):
     _fields_ = [("name", ctypes.c_char_p), ("n_stmts", ctypes.c_int32),
-                ("stmts", ctypes.POINTER(SpStmt))]
+                ("stmts", ctypes.POINTER(SpStmt)), ("box", ctypes.POINTER(ctypes.c_int64))]
 
 
 class SpArrayDesc(ctypes.Structure):
@@ -74,7 +74,9 @@ class SpGroupReport(ctypes.Structure):
                 ("flops_exec", ctypes.c_double), ("smem_bytes_pt", ctypes.c_double),
                 ("block_x", ctypes.c_int32), ("block_y", ctypes.c_int32),
                 ("block_cby", ctypes.c_int32), ("t_model_us", ctypes.c_double),
-                ("zqueue", ctypes.c_int32)]
+                ("zqueue", ctypes.c_int32), ("est_regs", ctypes.c_int32),
+                ("warmup_steps", ctypes.c_int32), ("prefetch", ctypes.c_int32),
+                ("instr_pt", ctypes.c_double)]
 
 
 # every symbol include/stencilfuse.h declares (checked by tests/test_abi.py)

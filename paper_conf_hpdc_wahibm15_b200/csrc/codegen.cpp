@@ -373,6 +373,14 @@ std::string generate_launch(const stencil_program *p, Launch &L, int index, bool
     o << "  const int cg = (Y0 + yt * VY + OYA) * XP + X0 + xt * VX + OXA;\n";
     o << "  const bool tile_in = X0 + TX <= NX && Y0 + TY <= NY;  // all core points interior\n";
 
+    // statement loop bounds (reading R2'): local-coordinate box of a boxed stage
+    std::set<int> box_cls;
+    auto sbox = [&](const Stage &G, int d) {
+        const Stmt &S = p->stmts[G.gid];
+        return d >= 4 ? S.box[d] - g.z_offset : S.box[d];
+    };
+    for (const Stage &G : L.st)
+        if (G.needed && p->stmts[G.gid].boxed) box_cls.insert(G.cls);
     // halo tables per class
     std::vector<int> nh(L.cls.size()), hp(L.cls.size());
     for (size_t c = 0; c < L.cls.size(); ++c) {
@@ -385,6 +393,8 @@ std::string generate_launch(const stencil_program *p, Launch &L, int index, bool
           << " per thread)\n";
         if (!nh[c]) continue;
         o << "  int h" << c << "_f[" << hp[c] << "], h" << c << "_g[" << hp[c] << "];\n";
+        if (box_cls.count((int)c))
+            o << "  int h" << c << "_x[" << hp[c] << "], h" << c << "_y[" << hp[c] << "];\n";
         for (const Lay &l : hlays[c]) o << "  int h" << c << "_" << lname(l) << "[" << hp[c] << "];\n";
         const int top = -R.y0, bot = R.y1, left = -R.x0, right = R.x1;
         o << "  #pragma unroll\n  for (int i = 0; i < " << hp[c] << "; ++i) {\n";
@@ -400,6 +410,7 @@ std::string generate_launch(const stencil_program *p, Launch &L, int index, bool
         o << "    h" << c << "_f[i] = ((gx >= 0 && gx < NX && gy >= 0 && gy < NY) ? 2 : 0)"
           << " | ((ax >= 0 && ax < XP && ay >= 0 && ay < YA) ? 8 : 0);\n";
         o << "    h" << c << "_g[i] = ay * XP + ax;\n";
+        if (box_cls.count((int)c)) o << "    h" << c << "_x[i] = gx; h" << c << "_y[i] = gy;\n";
         for (const Lay &l : hlays[c])
             o << "    h" << c << "_" << lname(l) << "[i] = (y - (" << ly0(l) << ")) * " << lw(l)
               << " + (x - (" << lx0(l) << "));\n";
@@ -596,11 +607,23 @@ std::string generate_launch(const stencil_program *p, Launch &L, int index, bool
         o << "      const int q = k + (" << G.lead << ");\n";
         o << "      if (q >= (" << G.loff << ") && q <= zc - 1 + (" << G.lead << ")) {\n";
         o << "        const int gz = Z0 + q;\n";
-        o << "        const bool zin = gz >= ZLO && gz < ZHI;\n";
+        const bool boxed = p->stmts[G.gid].boxed;
+        // in-box tests of this statement (the whole interior unless boxed)
+        const std::string BX0 = boxed ? num(sbox(G, 0)) : "0", BX1 = boxed ? num(sbox(G, 1)) : "NX";
+        const std::string BY0 = boxed ? num(sbox(G, 2)) : "0", BY1 = boxed ? num(sbox(G, 3)) : "NY";
+        if (boxed)
+            o << "        const bool zin = gz >= (" << sbox(G, 4) << ") && gz < (" << sbox(G, 5)
+              << ");  // loop bounds (R2')\n";
+        else
+            o << "        const bool zin = gz >= ZLO && gz < ZHI;\n";
         o << "        const bool zal = gz + OZA >= 0 && gz + OZA < ZA;\n";
         o << "        T *const gpl = p.arr[" << L.arr_slot[G.out] << "] + (long long)(gz + OZA) * PLANE;\n";
         if (G.stored) o << "        const bool zst = q >= 0 && q < zc;\n";
-        o << "        const bool fast = tile_in && zin;\n";
+        if (boxed)
+            o << "        const bool fast = X0 >= " << BX0 << " && X0 + TX <= " << BX1 << " && Y0 >= "
+              << BY0 << " && Y0 + TY <= " << BY1 << " && zin;\n";
+        else
+            o << "        const bool fast = tile_in && zin;\n";
 
         // ---- core blocks
         o << "        #pragma unroll\n        for (int b = 0; b < CBY; ++b) {\n";
@@ -728,7 +751,10 @@ std::string generate_launch(const stencil_program *p, Launch &L, int index, bool
         for (int iy = 0; iy < VY; ++iy)
             for (int jx = 0; jx < VX; ++jx) {
                 std::string gx = "X0 + xt * VX + " + num(jx), gy = "Y0 + by + " + num(iy);
-                o << "            if (!(zin && " << gx << " < NX && " << gy << " < NY)) o" << iy << "_"
+                const std::string inb = boxed ? gx + " >= " + BX0 + " && " + gx + " < " + BX1 +
+                                                    " && " + gy + " >= " + BY0 + " && " + gy + " < " + BY1
+                                              : gx + " < NX && " + gy + " < NY";
+                o << "            if (!(zin && " << inb << ")) o" << iy << "_"
                   << jx << " = sf_ldg_pred(gpl + cg + b * (YT * VY * XP) + (" << iy << " * XP + " << jx
                   << "), zal && " << gx << " < XP - OXA && " << gy << " < YA - OYA);\n";
             }
@@ -778,9 +804,15 @@ std::string generate_launch(const stencil_program *p, Launch &L, int index, bool
             o << "            } else {\n";
             for (int iy = 0; iy < VY; ++iy)
                 for (int jx = 0; jx < VX; ++jx)
-                    o << "              if (X0 + xt * VX + " << jx << " < NX && Y0 + by + " << iy
-                      << " < NY) sf_st(gb + (" << iy << " * XP + " << jx << "), o" << iy << "_" << jx
-                      << ");\n";
+                {
+                    const std::string gx = "X0 + xt * VX + " + num(jx), gy = "Y0 + by + " + num(iy);
+                    const std::string inb = boxed ? "zin && " + gx + " >= " + BX0 + " && " + gx + " < " +
+                                                        BX1 + " && " + gy + " >= " + BY0 + " && " + gy +
+                                                        " < " + BY1
+                                                  : gx + " < NX && " + gy + " < NY";
+                    o << "              if (" << inb << ") sf_st(gb + (" << iy << " * XP + " << jx
+                      << "), o" << iy << "_" << jx << ");\n";
+                }
             o << "            }\n          }\n";
         }
         o << "        }\n";
@@ -802,7 +834,12 @@ std::string generate_launch(const stencil_program *p, Launch &L, int index, bool
             o << "          const int f = h" << c << "_f[i];\n";
             // ghost points (e.g. the y-halo rows of full-height tiles) are only loaded
             o << "          T v;\n";
-            o << "          if (zin && (f & 2)) v = " << term_expr(halo_operand) << ";\n";
+            if (boxed)
+                o << "          const int hx = h" << c << "_x[i], hy = h" << c << "_y[i];\n"
+                  << "          if (zin && hx >= " << BX0 << " && hx < " << BX1 << " && hy >= " << BY0
+                  << " && hy < " << BY1 << ") v = " << term_expr(halo_operand) << ";\n";
+            else
+                o << "          if (zin && (f & 2)) v = " << term_expr(halo_operand) << ";\n";
             o << "          else v = sf_ldg_pred(gpl + h" << c << "_g[i], zal && (f & 8));\n";
             if (G.keep == Keep::Smem) {
                 Lay self{true, m};

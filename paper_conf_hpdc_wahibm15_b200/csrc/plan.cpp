@@ -171,6 +171,23 @@ static Launch analyze_group(const stencil_program *p, const std::vector<int> &me
         L.z_above = std::max(L.z_above, I.ahi);
     }
 
+    // R2' (loop bounds): a statement with a sub-box leaves the points outside its
+    // box to the array's stored value, which the fused kernel loads from memory;
+    // that is the value the original program sees only if no other statement of
+    // the group writes the array (before: the stored value would be stale; after:
+    // other CTAs would store there while this one loads)
+    for (int m = 0; m < n; ++m) {
+        const Stage &W = L.st[m];
+        if (!p->stmts[W.gid].boxed) continue;
+        for (int r = 0; r < n; ++r)
+            if (r != m && L.st[r].out == W.out)
+                fail(SP_E_PLAN_HAZARD,
+                     "statement " + std::to_string(W.gid) + " writes '" + p->arrays[W.out].name +
+                         "' over a sub-box of the interior and statement " +
+                         std::to_string(L.st[r].gid) + " of the same group also writes it "
+                         "(reading R2')");
+    }
+
     // R11: a group must not read from HBM an array it stores, except for a
     // point-wise read of the CTA's own tile and chunk that happens no later
     // than the store.
@@ -360,8 +377,8 @@ static void choose_config(const stencil_program *p, Launch &L, bool quick = fals
     else if (quick) cx = e == 8 ? std::vector<int>{32, 64} : std::vector<int>{64, 128};
     else cx = e == 8 ? std::vector<int>{16, 32, 64} : std::vector<int>{32, 64, 128};
     if (o.zchunk) cz = {o.zchunk};
-    else if (quick) cz = {16, 32, 64};
-    else cz = {4, 8, 16, 32, 64, 128, 256, 512};
+    else if (quick) cz = {16, 32};
+    else cz = {8, 16, 32};  // measured: longer chunks lose on every C2-C5 group (profiles/sweeps)
     if (o.threads) cn = {o.threads};
     else cn = {64, 128, 256};
     if (o.prefetch >= 0) cp = {o.prefetch};
@@ -374,7 +391,7 @@ static void choose_config(const stencil_program *p, Launch &L, bool quick = fals
     if (o.block_cby) ccb = {o.block_cby};
     else ccb = {1, 2, 4};
     const double sms = p->num_sms;
-    const double clk = 1.8e9;
+    const double clk = 1.85e9;
     const double hbm = 6.0e12, smem_bw = sms * 128 * clk;
     const double alu = sms * (e == 8 ? 64 : 128) * clk;
     const double pts = (double)g.nx * g.ny * nz;
@@ -422,25 +439,32 @@ static void choose_config(const stencil_program *p, Launch &L, bool quick = fals
                                     {(int64_t)(228 * 1024 / (C.smem + 1024)), (int64_t)(2048 / C.nth),
                                      32, (int64_t)(65536 / (C.nth * regs_alloc))});
                                 if (per_sm < 1) continue;
+                                // Launch-time model, fitted to measured sweeps of C2/C3/C4/C5
+                                // groups (tools/model_fit.py, profiles/sweeps/): the busiest
+                                // of HBM, shared memory (80 % of 128 B/clk/SM), FP pipe and
+                                // instruction issue, where issue is latency-limited by the
+                                // resident compute warps times the ILP of the register block;
+                                // HBM is latency-limited below ~1 us of bytes in flight per SM.
                                 double slots = sms * per_sm;
                                 double waves = std::ceil(ctas / slots);
                                 double fill = ctas / (waves * slots);
+                                const double res = std::min<double>(per_sm, std::ceil(ctas / sms));
                                 double t_mem = C.bytes_exec * pts / hbm;
-                                double t_sm = C.smem_pt * pts / smem_bw;
+                                double t_sm = C.smem_pt * pts / (smem_bw * 0.8);
                                 double t_alu = C.flops_exec * pts / alu;
-                                // issue rate: 4 warp-instructions per SM per cycle at ~70 %
-                                double t_issue = estimate_instr(C, p->opt.fmad && p->opt.factor) * pts / 32.0 / (sms * 4 * clk * 0.7);
-                                // latency hiding by the compute warps (barrier-separated stages)
-                                double warps = std::min<double>(per_sm, std::ceil(ctas / sms)) * nt / 32;
-                                double lat = std::min(1.0, warps / 16.0);
-                                double t = std::max({t_mem, t_sm / lat, t_alu / lat, t_issue / lat}) / fill;
-                                // bytes in flight per SM (TMA latency hiding): want >= 40 KB
-                                double inflight = 0;
-                                for (size_t i = 0; i < C.in.size(); ++i)
-                                    inflight += (double)C.in_rw[i] * C.in_rh[i] * e * pf;
-                                inflight *= std::min<double>(per_sm, std::ceil(ctas / sms));
-                                if (inflight < 40960) t *= std::sqrt(40960.0 / std::max(inflight, 1024.0));
-                                t += 2e-6 * waves;  // launch + wave tail overheads
+                                const double warps = res * nt / 32;
+                                const double ilp = std::min(4, vx * vy * cby);
+                                const double ipc = std::min(3.2, warps * std::sqrt(ilp) / 16.0);
+                                double t_issue = estimate_instr(C, p->opt.fmad && p->opt.factor) * pts /
+                                                 32.0 / (sms * ipc * clk);
+                                int n_store = 0;
+                                for (const Stage &G : C.st) n_store += G.needed && G.stored;
+                                const double inflight = res * (C.bytes_exec - n_store * e) * tx * ty *
+                                                        std::max(pf, 1);
+                                const double need = hbm / sms * 1e-6;
+                                if (inflight < need) t_mem *= need / std::max(inflight, 1.0);
+                                double t = std::max({t_mem, t_sm, t_alu, t_issue}) / fill;
+                                t += 100e-9 * (C.zc - C.kfirst) * waves;  // per-step march overhead
                                 C.t_model = t;
                                 if (t < best_t) { best_t = t; best = C; }
                             }
@@ -581,7 +605,10 @@ void fill_report(const stencil_program *p, const Launch &L, sp_group_report *r) 
     r->block_cby = L.cby;
     r->t_model_us = L.t_model * 1e6;
     r->zqueue = L.zq;
-    (void)p;
+    r->est_regs = L.est_regs;
+    r->warmup_steps = -L.kfirst;
+    r->prefetch = L.pf;
+    r->instr_pt = L.dead ? 0 : estimate_instr(L, p->opt.fmad && p->opt.factor);
 }
 
 }  // namespace sf

@@ -131,6 +131,19 @@ stencil_program *sf_program_create_impl(const sp_grid *grid, int32_t n_arrays,
         if (K.n_stmts <= 0 || !K.stmts) fail(SP_E_PROGRAM, "kernel without statements");
         Kernel kk;
         kk.name = K.name ? K.name : ("K" + std::to_string(k));
+        // loop bounds (R2'): default the whole global interior
+        int64_t box[6] = {0, g.nx, 0, g.ny, 0, g.nz_global};
+        bool boxed = false;
+        if (K.box) {
+            for (int d = 0; d < 6; ++d) box[d] = K.box[d];
+            for (int d = 0; d < 3; ++d) {
+                const int64_t hi = d == 0 ? g.nx : d == 1 ? g.ny : g.nz_global;
+                if (box[2 * d] < 0 || box[2 * d] > box[2 * d + 1] || box[2 * d + 1] > hi)
+                    fail(SP_E_PROGRAM, kk.name + ": box outside the interior or inverted");
+            }
+            boxed = box[0] != 0 || box[1] != g.nx || box[2] != 0 || box[3] != g.ny ||
+                    box[4] != 0 || box[5] != g.nz_global;
+        }
         std::vector<int> written;
         for (int s = 0; s < K.n_stmts; ++s) {
             const sp_stmt &S = K.stmts[s];
@@ -144,6 +157,8 @@ stencil_program *sf_program_create_impl(const sp_grid *grid, int32_t n_arrays,
             st.local = s;
             st.gid = gid++;
             st.out = S.out;
+            std::copy(box, box + 6, st.box);
+            st.boxed = boxed;
             for (int t = 0; t < S.n_terms; ++t) {
                 const sp_term &T = S.terms[t];
                 check_tap(p.get(), T.a, kk.name.c_str());

@@ -23,6 +23,8 @@ struct Stmt {
     int kernel, local, gid;  // kernel index, index inside kernel, global program-order id
     int out;
     std::vector<Term> terms;
+    int64_t box[6] = {0, 0, 0, 0, 0, 0};  // loop bounds, global interior coordinates (R2')
+    bool boxed = false;                   // box is smaller than the whole interior
 };
 struct Kernel { std::string name; std::vector<int> stmts; };
 struct ArrayDesc { std::string name; sp_role role; };

@@ -2,7 +2,8 @@
 
 It shares nothing with oracle.c: no loop nest, no index arithmetic — each term
 is a shifted NumPy view of the padded array.  Same reading of the paper as the
-oracle (R1-R4 in DESIGN.md): statements in program order, interior points only,
+oracle (R1-R4, R2' in DESIGN.md): statements in program order, interior points
+inside the kernel's loop bounds only,
 terms accumulated left to right in the program dtype, (c*a)*b for products.
 """
 import numpy as np
@@ -19,6 +20,8 @@ def run(prog, arrays):
         return a[hz + dz:hz + dz + nz, hy + dy:hy + dy + ny, hx + dx:hx + dx + nx]
 
     for k in prog["kernels"]:
+        # loop bounds (reading R2'): only the kernel's box of the interior is written
+        x0, x1, y0, y1, z0, z1 = k.get("box") or (0, nx, 0, ny, 0, nz)
         for s in k["stmts"]:
             acc = None
             for t in s["terms"]:
@@ -26,5 +29,5 @@ def run(prog, arrays):
                 if "b" in t:
                     v = v * view(*t["b"])
                 acc = v if acc is None else acc + v
-            view(s["out"], 0, 0, 0)[...] = acc
+            view(s["out"], 0, 0, 0)[z0:z1, y0:y1, x0:x1] = acc[z0:z1, y0:y1, x0:x1]
     return arrays

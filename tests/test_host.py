@@ -328,3 +328,48 @@ def test_wave_offsets_war_waw():
     p = Program(prog)
     p.set_plan([["K0"], ["K1"], ["K2"], ["K3"]])
     assert p.wave_offsets() == [0, 0, 2, 2]
+
+
+def test_fuzz_plans_legal_or_rejected_and_compile():
+    """Random legal programs (with and without loop bounds, R2') and random plans:
+    set_plan either accepts the plan or raises a plan error (never another failure),
+    and every accepted plan's kernels compile for sm_100a (NVRTC, no GPU needed)."""
+    import numpy as np
+    from _fuzz import random_lib_program, random_plans
+    accepted = rejected = 0
+    for seed in range(6):
+        rng = np.random.default_rng(seed)
+        prog = random_lib_program(rng, boxes=bool(seed % 2))
+        p = Program(prog)
+        p.compile("unfused")
+        for plan in random_plans(rng, prog, count=2):
+            try:
+                p.set_plan(plan)
+            except StencilError as e:
+                assert e.code in (4, 5, 6), e   # SP_E_PLAN_ORDER / _HAZARD / SP_E_RESOURCES
+                rejected += 1
+                continue
+            p.compile("fused")
+            accepted += 1
+    assert accepted > 0
+
+
+def test_box_validation_and_hazard():
+    T = P.tap
+    base = {"name": "b", "dtype": "f64", "grid": {"nx": 8, "ny": 6, "nz": 5, "ghost": [1, 1, 1]},
+            "arrays": [{"name": "A", "role": "in"}, {"name": "X", "role": "temp"},
+                       {"name": "O", "role": "out"}]}
+    k0 = {"name": "K0", "stmts": [{"out": "X", "terms": [{"c": 1.0, "a": T("A", (0, 0, 0))}]}]}
+    k1 = {"name": "K1", "box": [0, 8, 0, 6, 0, 1],
+          "stmts": [{"out": "X", "terms": [{"c": 2.0, "a": T("A", (0, 0, 1))}]}]}
+    k2 = {"name": "K2", "stmts": [{"out": "O", "terms": [{"c": 1.0, "a": T("X", (1, 0, 0))}]}]}
+    bad = dict(base, kernels=[dict(k1, box=[0, 9, 0, 6, 0, 1])])
+    with pytest.raises(StencilError) as e:
+        Program(bad)
+    assert e.value.code == 2                           # SP_E_PROGRAM: box beyond the interior
+    p = Program(dict(base, kernels=[k0, k1, k2]))
+    with pytest.raises(StencilError) as e:             # K0 and boxed K1 both write X in a group
+        p.set_plan([["K0", "K1", "K2"]])
+    assert "R2'" in str(e.value)
+    p.set_plan([["K0"], ["K1", "K2"]])                 # boxed writer alone in its group: fine
+    p.compile("fused")

@@ -225,7 +225,17 @@ def test_product_term_is_coef_times_a_times_b():
 
 
 # ------------------------------------------------------------- P5 independent evaluator
-def random_program(rng, dtype="f64"):
+def random_box(rng, n):
+    """Random loop bounds inside an interior of size n (possibly empty, possibly whole)."""
+    box = []
+    for d in range(3):
+        lo = int(rng.integers(0, n[d] + 1))
+        hi = int(rng.integers(lo, n[d] + 1))
+        box += [lo, hi]
+    return box
+
+
+def random_program(rng, dtype="f64", boxes=False):
     nx, ny, nz = (int(v) for v in rng.integers(1, 8, size=3))
     h = [2, 2, 2]
     n_arr = int(rng.integers(3, 7))
@@ -258,6 +268,8 @@ def random_program(rng, dtype="f64"):
                     if key in t and t[key][0] in wr:
                         t[key] = [t[key][0], 0, 0, 0]
         kernels.append({"name": f"K{kk}", "stmts": stmts})
+        if boxes and rng.random() < 0.6:
+            kernels[-1]["box"] = random_box(rng, (nx, ny, nz))
     return {"name": "rand", "dtype": dtype, "grid": {"nx": nx, "ny": ny, "nz": nz, "ghost": h},
             "arrays": [{"name": a, "role": r} for a, r in zip(names, roles)], "kernels": kernels}
 
@@ -353,3 +365,66 @@ def test_ghosts_never_written():
         m = np.ones(v.shape, bool)
         m[h:-h, h:-h, h:-h] = False
         assert np.array_equal(v[m], before[name][m]), name
+
+
+@pytest.mark.parametrize("seed", range(30))
+def test_p5_boxed_kernels_match_slicing_evaluator_bitexact(seed):
+    """Kernels with loop bounds (reading R2'): the oracle writes exactly the box."""
+    rng = np.random.default_rng(1000 + seed)
+    prog = random_program(rng, dtype="f64" if seed % 3 else "f32", boxes=True)
+    a1 = dense_arrays(prog, seed=seed)
+    a2 = {k: v.copy() for k, v in a1.items()}
+    OracleProgram(prog).run(a1)
+    _numpy_eval.run(prog, a2)
+    for name in a1:
+        assert a1[name].tobytes() == a2[name].tobytes(), name
+
+
+def _box_prog(box, terms, n=(6, 5, 4)):
+    return {"name": "box", "dtype": "f64",
+            "grid": {"nx": n[0], "ny": n[1], "nz": n[2], "ghost": [1, 1, 1]},
+            "arrays": [{"name": "A", "role": "in"}, {"name": "O", "role": "out"}],
+            "kernels": [{"name": "K", "box": box, "stmts": [{"out": "O", "terms": terms}]}]}
+
+
+def test_box_writes_exactly_the_box():
+    """O = 1*A over box [1,4)x[2,5)x[0,2) with A = 3 everywhere and O = -1: O is 3
+    exactly on the 3x3x2 box and keeps -1 everywhere else (ghosts included)."""
+    prog = _box_prog([1, 4, 2, 5, 0, 2], [{"c": 1.0, "a": ["A", 0, 0, 0]}])
+    arrs = {"A": np.full((6, 7, 8), 3.0), "O": np.full((6, 7, 8), -1.0)}
+    OracleProgram(prog).run(arrs)
+    O = arrs["O"]
+    inside = np.zeros_like(O, dtype=bool)
+    inside[1:3, 1 + 2:1 + 5, 1 + 1:1 + 4] = True
+    assert np.all(O[inside] == 3.0) and np.all(O[~inside] == -1.0)
+    assert inside.sum() == 18
+
+
+def test_box_boundary_plane_kernel_linear_field():
+    """A boundary kernel on the bottom plane only (k = 0): centred
+    difference in z of A = 2k + j gives 0.5*A[k+1] - 0.5*A[k-1] = 2 exactly there;
+    the other planes keep O = 0."""
+    n = (5, 4, 6)
+    prog = _box_prog([0, n[0], 0, n[1], 0, 1],
+                     [{"c": 0.5, "a": ["A", 0, 0, 1]}, {"c": -0.5, "a": ["A", 0, 0, -1]}], n)
+    k, j, i = np.meshgrid(np.arange(-1, n[2] + 1), np.arange(-1, n[1] + 1), np.arange(-1, n[0] + 1),
+                          indexing="ij")
+    arrs = {"A": np.ascontiguousarray(2.0 * k + j), "O": np.zeros(k.shape)}
+    OracleProgram(prog).run(arrs)
+    O = arrs["O"][1:-1, 1:-1, 1:-1]
+    assert np.all(O[0] == 2.0) and np.all(O[1:] == 0.0)
+
+
+def test_box_window_origin_translation():
+    """Evaluating a window of the grid with the window's global origin gives the
+    same points as the whole grid (statement boxes move with the window)."""
+    rng = np.random.default_rng(5)
+    prog = _box_prog([2, 5, 1, 4, 1, 3], [{"c": 0.25, "a": ["A", 1, 0, 0]},
+                                           {"c": 0.75, "a": ["A", 0, -1, 1]}])
+    full = dense_arrays(prog, seed=3)
+    ref = {k: v.copy() for k, v in full.items()}
+    OracleProgram(prog).run(ref)
+    # window: global interior x in [1,6), y in [0,5), z in [1,4) (with its ghosts)
+    win = {k: np.ascontiguousarray(v[1:6, 0:7, 1:8]) for k, v in full.items()}
+    OracleProgram(prog).run(win, n=(5, 5, 3), origin=(1, 0, 1))
+    assert np.array_equal(win["O"][1:-1, 1:-1, 1:-1], ref["O"][2:5, 1:6, 2:7])

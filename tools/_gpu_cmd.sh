@@ -1,4 +1,4 @@
 export PYTHONUNBUFFERED=1
-timeout 700 python tools/sweep.py C4 --group 2 --grid --tx 32,64,128,256 --zchunk 32 --pf 1,2,3 > gpurun_out/sw2_g2.log 2>&1
-timeout 700 python tools/sweep.py C4 --group 5 --grid --tx 32,64,128 --zchunk 32 --pf 2,3 > gpurun_out/sw2_g5.log 2>&1
-tail -3 gpurun_out/sw2_g2.log
+timeout 900 python tools/sweep.py C2 --group 0 --grid --tx 32,64 --zchunk 8,16,32,64 --pf 2 > gpurun_out/sw_c2.log 2>&1
+timeout 900 python tools/sweep.py C3 --plan-name fission_fused --group 0 --grid --tx 64,128 --zchunk 8,16,32 --pf 2 > gpurun_out/sw_c3.log 2>&1
+timeout 900 python tools/sweep.py C5 --group 0 --grid --tx 32,64 --zchunk 8,16,32 --pf 2 > gpurun_out/sw_c5.log 2>&1

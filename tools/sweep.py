@@ -23,10 +23,11 @@ def main():
     ap.add_argument("--group", type=int, default=0)
     ap.add_argument("--mode", default="fused")
     ap.add_argument("--plan", default=None)
+    ap.add_argument("--plan-name", default="fused", help="named plan of the workload")
     ap.add_argument("--cfg", action="append", default=[])
     ap.add_argument("--iters", type=int, default=10)
     ap.add_argument("--grid", action="store_true", help="enumerate tile/block combinations")
-    ap.add_argument("--zchunk", type=int, default=32)
+    ap.add_argument("--zchunk", default="32", help="comma list of z-chunk lengths")
     ap.add_argument("--tx", default="32,64")
     ap.add_argument("--pf", default="", help="comma list of prefetch depths to cross with --grid")
     ap.add_argument("--apply-tuning", action="store_true", help="pin the plan's tuned configs first")
@@ -43,18 +44,19 @@ def main():
                             ty = nt // xt * by * cb
                             if ty > 32:
                                 continue
-                            c = (f"tile_x={tx},block_x={bx},threads={nt},block_y={by},"
-                                 f"block_cby={cb},tile_y={ty},zchunk={a.zchunk}")
-                            if a.pf:
-                                a.cfg += [c + f",prefetch={pf}" for pf in a.pf.split(",")]
-                            else:
-                                a.cfg.append(c)
+                            for zc in a.zchunk.split(","):
+                                c = (f"tile_x={tx},block_x={bx},threads={nt},block_y={by},"
+                                     f"block_cby={cb},tile_y={ty},zchunk={zc}")
+                                if a.pf:
+                                    a.cfg += [c + f",prefetch={pf}" for pf in a.pf.split(",")]
+                                else:
+                                    a.cfg.append(c)
     if a.workload.startswith("probe:"):
         from probe_programs import probe
         prog = probe(a.workload)
     else:
         prog = bench.load_workload(a.workload)
-    plan = json.load(open(a.plan))["groups"] if a.plan else bench.plan_of(prog)
+    plan = json.load(open(a.plan))["groups"] if a.plan else bench.plan_of(prog, a.plan_name)
     dev = torch.device("cuda:0")
     flush = torch.ones(32 << 20, dtype=torch.float64, device=dev)  # read-only L2 flush (no dirty lines)
     base = None

@@ -32,6 +32,11 @@ UNIT = "grid-point updates/s"
 
 
 def load_workload(name):
+    """Program dict of a workload.  Frozen plans and tuned per-launch configurations
+    (measured on B200 with tools/ab_plans.py / tools/step_tune.py) come from
+    configs/<workload>_plan.json: C4's plan is the measured-greedy planner output;
+    the other workloads keep their hand plans (synth/programs.py) and only carry
+    configurations, keyed by plan name."""
     from synth import programs as P
     if name == "C4":
         from synth.scale_les import c4
@@ -41,17 +46,25 @@ def load_workload(name):
         if os.path.exists(plan_path):
             pj = json.load(open(plan_path))
             prog["plans"]["fused"] = pj["groups"]
-            prog["plan_configs"] = pj.get("configs")
+            prog["plan_configs"] = {"fused": pj.get("configs")}
         return prog
-    return P.CONFIGS[name]()
+    prog = P.CONFIGS[name]()
+    path = os.path.join(ROOT, "configs", f"{name.lower()}_plan.json")
+    if os.path.exists(path):
+        pj = json.load(open(path))
+        prog["plan_configs"] = {k: v.get("configs") for k, v in pj["plans"].items()}
+        for k, v in pj["plans"].items():  # searched plans (e.g. "measured") carry their groups
+            if v.get("groups"):
+                prog["plans"][k] = v["groups"]
+    return prog
 
 
-def tuned_configs(prog):
-    return prog.get("plan_configs")
+def tuned_configs(prog, plan="fused"):
+    return (prog.get("plan_configs") or {}).get(plan)
 
 
-def apply_tuning(p, prog):
-    cfgs = tuned_configs(prog)
+def apply_tuning(p, prog, plan="fused"):
+    cfgs = tuned_configs(prog, plan)
     if cfgs:
         for i, c in enumerate(cfgs):
             if c:
@@ -156,14 +169,14 @@ def run_ours(args):
     # deep halo needed by the plan's accumulated z-reach (probe on the local grid)
     probe = Program(prog)
     probe.set_plan(plan)
-    apply_tuning(probe, prog)
+    apply_tuning(probe, prog, args.plan)
     reach = max([max(r["z_below"], r["z_above"]) for r in probe.reports("fused")] + [prog["grid"]["ghost"][2]])
     zhalo = reach if world > 1 else prog["grid"]["ghost"][2]
     del probe
     comm = Comm(rank, world) if world > 1 else None
     p = Program(prog, comm=comm, nz_global=nz * world, z_offset=rank * nz, zhalo=zhalo)
     p.set_plan(plan)
-    apply_tuning(p, prog)
+    apply_tuning(p, prog, args.plan)
     p.allocate(dev, fill=0.0)
     fill_inputs(p, prog, dev, rank * nz, zhalo)
     stream = torch.cuda.current_stream(dev)

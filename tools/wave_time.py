@@ -22,9 +22,10 @@ def main():
     ap.add_argument("--waves", nargs="+", default=["0:1", "32:2", "64:2"])
     ap.add_argument("--steps", type=int, default=100)
     ap.add_argument("--opt", action="append", default=[])
+    ap.add_argument("--plan", default="fused", help="named plan (e.g. unfused: one group per kernel)")
     a = ap.parse_args()
     prog = bench.load_workload(a.workload)
-    plan = bench.plan_of(prog)
+    plan = bench.plan_of(prog, a.plan)
     dev = torch.device("cuda:0")
     stream = torch.cuda.current_stream(dev)
     pts = prog["grid"]["nx"] * prog["grid"]["ny"] * prog["grid"]["nz"]
@@ -36,7 +37,8 @@ def main():
         zw, ns = (int(v) for v in spec.split(":"))
         p = Program(prog, options=dict(extra, zwave=zw, zwave_streams=ns))
         p.set_plan(plan)
-        bench.apply_tuning(p, prog)
+        if a.plan == "fused":
+            bench.apply_tuning(p, prog)
         if base is None:
             p.allocate(dev, fill=0.0)
             bench.fill_inputs(p, prog, dev, 0, prog["grid"]["ghost"][2])
@@ -63,7 +65,7 @@ def main():
         torch.cuda.synchronize()
         ms = s.elapsed_time(e) / a.steps
         alg = sum(r["bytes_alg"] for r in p.reports("fused")) * pts
-        print(f"zwave {zw:4d} streams {ns}: {ms:.4f} ms/step  {alg / ms / 1e6:7.0f} GB/s alg  "
+        print(f"{a.plan} zwave {zw:4d} streams {ns}: {ms:.4f} ms/step  {alg / ms / 1e6:7.0f} GB/s alg  "
               f"{pts * len(prog['kernels']) / ms / 1e6:.3e} upd/s  bit-exact {exact}", flush=True)
         del p
 

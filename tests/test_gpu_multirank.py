@@ -48,7 +48,16 @@ def plane(p, t, z, depth):
     return t[oz + z:oz + z + depth]
 
 
-@pytest.mark.parametrize("cfg,ranks", [("C2", 2), ("C5", 3), ("C3", 2), ("C4", 2), ("chain3", 3)])
+def c2_boxed(nz):
+    """C2 whose update kernel has loop bounds (reading R2') crossing the slab boundary
+    (global z in [5, 20) for 2 x 12 planes), so boxed stages meet deep-halo planes."""
+    prog = P.c2(nx=40, ny=24, nz=nz)
+    prog["kernels"][3]["box"] = [3, 30, 2, 20, 5, 20]
+    return prog
+
+
+@pytest.mark.parametrize("cfg,ranks", [("C2", 2), ("C5", 3), ("C3", 2), ("C4", 2), ("chain3", 3),
+                                       ("C2box", 2)])
 @pytest.mark.parametrize("fmad", [0, 1])
 def test_virtual_ranks_bitexact(cuda_device, cfg, ranks, fmad):
     import torch
@@ -56,7 +65,7 @@ def test_virtual_ranks_bitexact(cuda_device, cfg, ranks, fmad):
     nzl = 12
     mk = {"C2": lambda nz: P.c2(nx=40, ny=24, nz=nz), "C5": lambda nz: P.c5(nx=32, ny=16, nz=nz),
           "C3": lambda nz: P.c3(nx=48, ny=20, nz=nz), "C4": c4_small,
-          "chain3": lambda nz: P.resize(P.chain3(), 20, 12, nz)}[cfg]
+          "chain3": lambda nz: P.resize(P.chain3(), 20, 12, nz), "C2box": c2_boxed}[cfg]
     glob = mk(nzl * ranks)
     plan = glob["plans"]["fused"]
     opts = {"fmad": fmad}
@@ -69,7 +78,7 @@ def test_virtual_ranks_bitexact(cuda_device, cfg, ranks, fmad):
     single.run_fused()
     # slabs
     loc = mk(nzl)
-    probe = Program(loc, options=opts)
+    probe = Program(loc, nz_global=nzl * ranks, options=opts)
     probe.set_plan(plan)
     zhalo = max([max(r["z_below"], r["z_above"]) for r in probe.reports("fused")] +
                 [loc["grid"]["ghost"][2]])

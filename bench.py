@@ -170,7 +170,8 @@ def run_ours(args):
     probe = Program(prog)
     probe.set_plan(plan)
     apply_tuning(probe, prog, args.plan)
-    reach = max([max(r["z_below"], r["z_above"]) for r in probe.reports("fused")] + [prog["grid"]["ghost"][2]])
+    reach = max([max(r["z_below"], r["z_above"]) for m in ("fused", "unfused") for r in probe.reports(m)] +
+                [prog["grid"]["ghost"][2]])
     zhalo = reach if world > 1 else prog["grid"]["ghost"][2]
     del probe
     comm = Comm(rank, world) if world > 1 else None
@@ -350,7 +351,9 @@ def run_ours(args):
                                  "predicted_traffic_reduction": 1 - alg_step / alg_step_u},
             "e2e": {"value": updates / (e2e_ms * 1e-3), "unit": UNIT, "h2d_bytes_per_step": h2d,
                     "d2h_bytes_per_step": d2h, "ms_per_step": e2e_ms},
-            "gpu_launches": args.steps * len(live_f),
+            # N > 1: a launch that receives ghost planes runs as interior + 2 boundary launches
+            "gpu_launches": args.steps * sum(3 if world > 1 and p.exchange_plan("fused", i) else 1
+                                             for i in live_f),
             "clocks": clocks,
             "wall_s_timed": wall,
         }

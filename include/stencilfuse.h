@@ -157,6 +157,15 @@ typedef struct stencil_program_s stencil_program;
  * device of the calling thread is used.  Collective over nranks. */
 sp_status sp_comm_unique_id(void *out128);
 sp_status sp_comm_create(const void *nccl_unique_id, int32_t nranks, int32_t rank, sp_comm **out);
+/* Test transport: nranks communicators (out[0..nranks-1]) of in-process virtual
+ * ranks on the current device.  Each virtual rank's program must be driven from
+ * its own host thread (the exchanges meet at host barriers, 120 s timeout ->
+ * SP_E_STATE); ghost planes are pulled from the neighbours' bound slabs with
+ * device-to-device copies on the comm stream, ordered by events, in place of
+ * ncclSend/ncclRecv.  Every other step of the multi-rank schedule (exchange set,
+ * interior/boundary planes, events) is the NCCL path's.  Destroy each with
+ * sp_comm_destroy. */
+sp_status sp_comm_create_loopback(int32_t nranks, sp_comm **out);
 void sp_comm_destroy(sp_comm *comm);
 
 /* ---- program ------------------------------------------------------------ */
@@ -248,12 +257,17 @@ typedef struct {
  * configuration does not fit. */
 sp_status sp_plan_tune(stencil_program *prog, int32_t mode, int32_t launch, const sp_tile_config *cfg);
 
-/* Halo-exchange schedule of one launch on several ranks: the arrays it reads
- * beyond the local slab (up to cap written to arrays[], *n = total) and the
- * exchange depth (its accumulated z reach, <= zhalo).  run_fused performs
- * exactly this exchange before the launch's boundary chunks. */
+/* Halo-exchange schedule of one launch on several ranks: the
+ * arrays whose ghost planes are received right before it (up to cap written to
+ * arrays[], *n = total), with the planes received into the bottom ghost
+ * (below[i]) and the top ghost (above[i]); below/above may be NULL.  An array
+ * is received once per epoch (step start, or a launch that stores it, up to the
+ * next), before the epoch's first launch that reads it beyond the slab, at the
+ * largest depth any reader of the epoch needs (each <= zhalo).  run_unfused /
+ * run_fused perform exactly this exchange, overlapped with the launch's
+ * interior planes; host-only (no GPU needed). */
 sp_status sp_plan_exchange(stencil_program *prog, int32_t mode, int32_t launch, int32_t cap,
-                           int32_t *arrays, int32_t *n, int32_t *depth);
+                           int32_t *arrays, int32_t *below, int32_t *above, int32_t *n);
 /* z-wave schedule of the fused mode (options "zwave" = S planes per wave,
  * "zwave_streams" = waves in flight on that many streams; single rank only).
  * In wave w, launch i evaluates output planes [w*S - off_i, (w+1)*S - off_i)
@@ -272,8 +286,9 @@ sp_status sp_compile(stencil_program *prog, int32_t mode);
  * reading its inputs from and writing all its outputs to HBM. */
 sp_status run_unfused(stencil_program *prog, sp_stream stream);
 /* The current plan's groups in order (SP_E_STATE if no plan).  On several
- * ranks each group is preceded by the halo exchange its z-reach needs,
- * overlapped with the group's interior chunks. */
+ * ranks a group whose schedule (sp_plan_exchange) receives ghost planes runs
+ * its interior planes while the exchange is in flight on the communicator's
+ * stream, then its boundary planes. */
 sp_status run_fused(stencil_program *prog, sp_stream stream);
 /* One launch of a mode (profiling / per-kernel timing); no exchange. */
 sp_status sp_run_launch(stencil_program *prog, int32_t mode, int32_t launch, sp_stream stream);

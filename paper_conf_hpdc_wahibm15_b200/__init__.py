@@ -61,6 +61,20 @@ class Comm:
         _check(lib().sp_comm_create(raw, world, rank, ctypes.byref(self.handle)))
         self.rank, self.world = rank, world
 
+    @classmethod
+    def loopback(cls, world: int):
+        """Test transport: `world` in-process virtual ranks on the current device
+        (sp_comm_create_loopback).  Drive each rank's Program from its own thread."""
+        hs = (ctypes.c_void_p * world)()
+        _check(lib().sp_comm_create_loopback(world, hs))
+        out = []
+        for r in range(world):
+            c = cls.__new__(cls)
+            c.handle = ctypes.c_void_p(hs[r])
+            c.rank, c.world = r, world
+            out.append(c)
+        return out
+
     def __del__(self):
         h = getattr(self, "handle", None)
         if h:
@@ -276,12 +290,14 @@ class Program:
         _check(lib().sp_plan_tune(self.handle, self._mode(mode), i, ctypes.byref(c)))
 
     def exchange_plan(self, mode, i):
-        """(array names, depth) the executor exchanges before launch i on several ranks."""
-        n, depth = ctypes.c_int32(), ctypes.c_int32()
-        buf = (ctypes.c_int32 * len(self.names))()
-        _check(lib().sp_plan_exchange(self.handle, self._mode(mode), i, len(self.names), buf,
-                                      ctypes.byref(n), ctypes.byref(depth)))
-        return [self.names[buf[j]] for j in range(n.value)], depth.value
+        """[(array name, planes below, planes above)] the executor receives into the
+        ghost planes right before launch i on several ranks (sp_plan_exchange)."""
+        n = ctypes.c_int32()
+        k = len(self.names)
+        buf, lo, hi = (ctypes.c_int32 * k)(), (ctypes.c_int32 * k)(), (ctypes.c_int32 * k)()
+        _check(lib().sp_plan_exchange(self.handle, self._mode(mode), i, k, buf, lo, hi,
+                                      ctypes.byref(n)))
+        return [(self.names[buf[j]], lo[j], hi[j]) for j in range(n.value)]
 
     def wave_offsets(self):
         """Plane skew of each fused launch in the z-wave schedule (option "zwave")."""

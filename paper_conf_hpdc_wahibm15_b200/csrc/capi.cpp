@@ -19,6 +19,7 @@ void sf_unfused_prepare(stencil_program *);
 sp_comm *sf_comm_create_impl(const void *, int32_t, int32_t);
 void sf_comm_destroy_impl(sp_comm *);
 void sf_comm_unique_id_impl(void *);
+void sf_comm_create_loopback_impl(int32_t, sp_comm **);
 
 namespace sf {
 static thread_local std::string t_err;
@@ -61,28 +62,20 @@ static Mode &mode_of(stencil_program *p, int mode) {
     fail(SP_E_ARG, "mode must be 0 (unfused) or 1 (fused)");
 }
 
-// chunks of launch L whose reads stay inside the local slab (no ghost planes
-// exchanged by this group needed): [lo, hi)
-static void interior_chunks(const stencil_program *p, const Launch &L, int *lo, int *hi) {
-    const int64_t nz = p->grid.nz_local;
-    int qlo = 0, ahi = 0;
-    for (const Input &I : L.in) { qlo = std::min(qlo, I.qlo); ahi = std::max(ahi, I.ahi); }
-    int a = L.nch, b = 0;
-    for (int c = 0; c < L.nch; ++c) {
-        int64_t z0 = (int64_t)c * L.zc, z1 = std::min<int64_t>(z0 + L.zc, nz);
-        if (z0 + qlo >= 0 && z1 - 1 + ahi <= nz - 1) { a = std::min(a, c); b = std::max(b, c + 1); }
-    }
-    if (a >= b) { a = 0; b = 0; }
-    *lo = a;
-    *hi = b;
-}
-
-// inputs a launch reads beyond the local slab, and the exchange depth (its z reach)
-static int exchange_set(const Launch &L, std::vector<int> &arrays) {
-    arrays.clear();
-    for (const Input &I : L.in)
-        if (I.qlo < 0 || I.ahi > 0) arrays.push_back(I.arr);
-    return std::max(L.z_below, L.z_above);
+// output planes [*zb, *ze) of launch L that read no ghost plane received by the
+// exchange in front of it: they run while the exchange is in flight
+static void interior_planes(const stencil_program *p, const Launch &L,
+                            const std::vector<Mode::Xfer> &x, int *zb, int *ze) {
+    const int nz = (int)p->grid.nz_local;
+    int b = 0, e = nz;
+    for (const Mode::Xfer &t : x)
+        for (const Input &I : L.in)
+            if (I.arr == t.arr) {
+                b = std::max(b, -I.qlo);
+                e = std::min(e, nz - std::max(0, I.ahi));
+            }
+    *zb = b;
+    *ze = e;
 }
 
 // ---------------------------------------------------------------- z-wave schedule
@@ -197,38 +190,55 @@ static void run_mode(stencil_program *p, int mode, void *stream) {
         run_waves(p, m, stream);
         return;
     }
+    if (!multi) {
+        for (size_t i = 0; i < m.launches.size(); ++i) launch(p, m, (int)i, stream, 0, 1, m.launches[i].nch);
+        return;
+    }
+    // several ranks: programmatic dependent launch is not used across the exchange's
+    // events (launch() sees p->no_pdl); each launch whose schedule receives ghost
+    // planes runs its interior planes while the exchange is in flight, then the
+    // boundary planes (a few planes each) once the ghosts have arrived
+    if (!m.xsched_ok) exchange_schedule(p, m);
+    p->no_pdl = true;
+    const int nz = (int)p->grid.nz_local;
+    cudaStream_t cs = (cudaStream_t)p->comm->comm_stream;
+    while (p->events.size() < 2) {
+        cudaEvent_t ev;
+        if (cudaEventCreateWithFlags(&ev, cudaEventDisableTiming) != cudaSuccess)
+            fail(SP_E_CUDA, "cudaEventCreate");
+        p->events.push_back(ev);
+    }
+    cudaEvent_t ready = (cudaEvent_t)p->events[0], done = (cudaEvent_t)p->events[1];
+    auto planes = [&](int i, int z0, int z1) {
+        const int zc = m.launches[i].zc;
+        if (z1 > z0) launch(p, m, i, stream, 0, 1, (z1 - z0 + zc - 1) / zc, z0, z1);
+    };
     for (size_t i = 0; i < m.launches.size(); ++i) {
         Launch &L = m.launches[i];
         if (L.dead) continue;
-        std::vector<int> xarr;
-        int depth = exchange_set(L, xarr);
-        if (!multi || depth == 0 || xarr.empty()) {
-            launch(p, m, (int)i, stream, 0, 1, L.nch);
+        const std::vector<Mode::Xfer> &x = m.xsched[i];
+        if (x.empty()) {
+            planes((int)i, 0, nz);
             continue;
         }
-        int lo, hi;
-        interior_chunks(p, L, &lo, &hi);
+        int zb, ze;
+        interior_planes(p, L, x, &zb, &ze);
         // exchange on the communicator's stream, ordered after prior work on `stream`
-        cudaStream_t cs = (cudaStream_t)p->comm->comm_stream;
-        if (p->events.size() < 2) {
-            for (int e = 0; e < 2; ++e) {
-                cudaEvent_t ev;
-                if (cudaEventCreateWithFlags(&ev, cudaEventDisableTiming) != cudaSuccess)
-                    fail(SP_E_CUDA, "cudaEventCreate");
-                p->events.push_back(ev);
-            }
-        }
-        cudaEvent_t ready = (cudaEvent_t)p->events[0], done = (cudaEvent_t)p->events[1];
         if (cudaEventRecord(ready, (cudaStream_t)stream) != cudaSuccess ||
             cudaStreamWaitEvent(cs, ready, 0) != cudaSuccess)
             fail(SP_E_CUDA, "event record/wait");
-        exchange(p, xarr, depth, cs);
+        exchange(p, x, cs);
         if (cudaEventRecord(done, cs) != cudaSuccess) fail(SP_E_CUDA, "event record");
-        if (hi > lo) launch(p, m, (int)i, stream, lo, 1, hi - lo);   // interior: overlaps
+        const bool split = ze > zb;
+        if (split) planes((int)i, zb, ze);  // interior: overlaps the exchange
         if (cudaStreamWaitEvent((cudaStream_t)stream, done, 0) != cudaSuccess)
             fail(SP_E_CUDA, "stream wait");
-        if (lo > 0) launch(p, m, (int)i, stream, 0, 1, lo);
-        if (hi < L.nch) launch(p, m, (int)i, stream, hi, 1, L.nch - hi);
+        if (split) {
+            planes((int)i, 0, zb);
+            planes((int)i, ze, nz);
+        } else {
+            planes((int)i, 0, nz);
+        }
     }
 }
 
@@ -247,6 +257,13 @@ sp_status sp_comm_create(const void *id, int32_t nranks, int32_t rank, sp_comm *
     return guard([&] {
         if (!id || !out || nranks < 1 || rank < 0 || rank >= nranks) fail(SP_E_ARG, "bad comm args");
         *out = sf_comm_create_impl(id, nranks, rank);
+    });
+}
+
+sp_status sp_comm_create_loopback(int32_t nranks, sp_comm **out) {
+    return guard([&] {
+        if (!out || nranks < 1) fail(SP_E_ARG, "bad loopback args");
+        sf_comm_create_loopback_impl(nranks, out);
     });
 }
 
@@ -457,15 +474,19 @@ sp_status sp_plan_tune(stencil_program *p, int32_t mode, int32_t launch, const s
 }
 
 sp_status sp_plan_exchange(stencil_program *p, int32_t mode, int32_t launch, int32_t cap,
-                           int32_t *arrays, int32_t *n, int32_t *depth) {
+                           int32_t *arrays, int32_t *below, int32_t *above, int32_t *n) {
     return guard([&] {
-        if (!p || !n || !depth) fail(SP_E_ARG, "null argument");
+        if (!p || !n || (cap > 0 && !arrays)) fail(SP_E_ARG, "null argument");
         Mode &m = mode_of(p, mode);
         if (launch < 0 || launch >= (int)m.launches.size()) fail(SP_E_ARG, "launch index out of range");
-        std::vector<int> a;
-        *depth = m.launches[launch].dead ? 0 : exchange_set(m.launches[launch], a);
-        *n = (int)a.size();
-        for (int i = 0; i < std::min<int>(cap, (int)a.size()); ++i) arrays[i] = a[i];
+        if (!m.xsched_ok) exchange_schedule(p, m);
+        const std::vector<Mode::Xfer> &x = m.xsched[launch];
+        *n = (int)x.size();
+        for (int i = 0; i < std::min<int>(cap, (int)x.size()); ++i) {
+            arrays[i] = x[i].arr;
+            if (below) below[i] = x[i].below;
+            if (above) above[i] = x[i].above;
+        }
     });
 }
 
@@ -517,10 +538,12 @@ sp_status exchange_halos(stencil_program *p, int32_t n, const int32_t *arrays, i
         if (!p->comm) fail(SP_E_STATE, "exchange_halos needs a communicator");
         if (depth < 1 || depth > p->grid.zhalo || depth > p->grid.nz_local)
             fail(SP_E_ARG, "depth must be in [1, min(zhalo, nz_local)]");
-        std::vector<int> a(arrays, arrays + n);
-        for (int x : a)
-            if (x < 0 || x >= (int)p->arrays.size()) fail(SP_E_ARG, "bad array index");
-        exchange(p, a, depth, stream);
+        std::vector<Mode::Xfer> x;
+        for (int i = 0; i < n; ++i) {
+            if (arrays[i] < 0 || arrays[i] >= (int)p->arrays.size()) fail(SP_E_ARG, "bad array index");
+            x.push_back({arrays[i], depth, depth});
+        }
+        exchange(p, x, stream);
     });
 }
 

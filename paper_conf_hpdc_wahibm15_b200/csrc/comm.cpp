@@ -1,13 +1,23 @@
-// comm.cpp — z-slab halo exchange over NCCL (new relative to the
-// paper, which runs on a single node, §6.1.2).
+// comm.cpp — z-slab halo exchange (new relative to the paper,
+// which runs on a single node, §6.1.2).
 //
 // Rank r owns global planes [z_offset, z_offset + nz_local).  Ghost planes are
-// contiguous because z is the slowest axis, so each direction is one
-// ncclSend/ncclRecv of depth * plane elements, with no packing.  All arrays of
-// one exchange go in one ncclGroupStart/End.
+// contiguous because z is the slowest axis, so each direction is one transfer of
+// depth * plane elements per array, with no packing.  Two transports:
+//   * NCCL (one process per GPU): ncclSend/ncclRecv, all arrays of one exchange
+//     in one ncclGroupStart/End;
+//   * loopback (test transport): the virtual ranks of one process on one device,
+//     each driven from its own host thread; a rank pulls its ghost planes from the
+//     neighbours' slabs with device-to-device copies, ordered by events that the
+//     ranks publish at host barriers.  It runs the executor's multi-rank schedule
+//     (exchange set, interior/boundary split, events) exactly as NCCL does; only
+//     the wire differs.
 #include <cuda_runtime.h>
 #include <nccl.h>
 
+#include <algorithm>
+#include <chrono>
+#include <condition_variable>
 #include <cstring>
 
 #include "sf_internal.h"
@@ -17,11 +27,162 @@ static void nccl_check(ncclResult_t r, const char *what) {
         sf::fail(SP_E_NCCL, std::string(what) + ": " + ncclGetErrorString(r));
 }
 
+namespace sf {
+
+struct LoopHub {
+    int n = 0;
+    std::mutex mu;
+    std::condition_variable cv;
+    int arrived = 0;
+    uint64_t gen = 0;
+    std::vector<stencil_program *> prog;
+    std::vector<cudaEvent_t> ready, done;
+
+    // all n virtual ranks meet; a missing rank (an error on its thread) times out
+    void barrier() {
+        std::unique_lock<std::mutex> lk(mu);
+        const uint64_t g = gen;
+        if (++arrived == n) {
+            arrived = 0;
+            ++gen;
+            cv.notify_all();
+            return;
+        }
+        if (!cv.wait_for(lk, std::chrono::seconds(120), [&] { return gen != g; })) {
+            --arrived;
+            fail(SP_E_STATE, "loopback exchange: a virtual rank did not reach the exchange "
+                             "(each rank must run the same plan on its own host thread)");
+        }
+    }
+    ~LoopHub() {
+        for (cudaEvent_t e : ready) cudaEventDestroy(e);
+        for (cudaEvent_t e : done) cudaEventDestroy(e);
+    }
+};
+
+// Per launch, the arrays whose ghost planes must be received before it, with the
+// depth below/above.  An array is exchanged once per "epoch" (the step start or a
+// launch that stores it, up to the next such launch), before the epoch's first
+// launch that reads it beyond the slab, at the largest depth any reader of the
+// epoch needs; an unchanged array is not re-sent to every consumer.  A launch
+// never reads beyond the slab an array it stores (reading R11), so the epoch's
+// value is the one every reader sees.
+void exchange_schedule(const stencil_program *p, Mode &m) {
+    const size_t n = m.launches.size();
+    const int na = (int)p->arrays.size();
+    m.xsched.assign(n, {});
+    std::vector<int> first(na, -1), below(na, 0), above(na, 0);
+    auto flush = [&](int a) {
+        if (first[a] >= 0) m.xsched[first[a]].push_back({a, below[a], above[a]});
+        first[a] = -1;
+        below[a] = above[a] = 0;
+    };
+    for (size_t i = 0; i < n; ++i) {
+        const Launch &L = m.launches[i];
+        if (L.dead) continue;
+        for (const Input &I : L.in) {
+            const int b = std::max(0, -I.qlo), u = std::max(0, I.ahi);
+            if (!b && !u) continue;
+            if (first[I.arr] < 0) first[I.arr] = (int)i;
+            below[I.arr] = std::max(below[I.arr], b);
+            above[I.arr] = std::max(above[I.arr], u);
+        }
+        for (const Stage &G : L.st)
+            if (G.stored) flush(G.out);
+    }
+    for (int a = 0; a < na; ++a) flush(a);
+    for (auto &v : m.xsched)
+        std::sort(v.begin(), v.end(), [](const Mode::Xfer &x, const Mode::Xfer &y) { return x.arr < y.arr; });
+    m.xsched_ok = true;
+}
+
+static void exchange_loopback(stencil_program *p, const std::vector<Mode::Xfer> &x,
+                              cudaStream_t s) {
+    sp_comm *c = p->comm;
+    LoopHub &h = *c->hub;
+    const int r = c->rank;
+    h.prog[r] = p;
+    if (cudaEventRecord(h.ready[r], s) != cudaSuccess) fail(SP_E_CUDA, "event record");
+    h.barrier();  // every rank's slab is final up to its `ready`
+    const int up = r + 1 < h.n ? r + 1 : -1, dn = r > 0 ? r - 1 : -1;
+    for (int nb : {up, dn})
+        if (nb >= 0 && cudaStreamWaitEvent(s, h.ready[nb], 0) != cudaSuccess)
+            fail(SP_E_CUDA, "stream wait");
+    const int64_t nz = p->grid.nz_local;
+    const size_t pb = (size_t)(p->plane * p->elem);
+    for (const Mode::Xfer &t : x) {
+        auto at = [&](stencil_program *q, int64_t z) {
+            if (!q->ptrs[t.arr]) fail(SP_E_STATE, "array '" + q->arrays[t.arr].name + "' is not bound");
+            return (char *)q->ptrs[t.arr] + (z + q->layout.origin_z) * pb;
+        };
+        if (up >= 0 && t.above > 0 &&
+            cudaMemcpyAsync(at(p, nz), at(h.prog[up], 0), t.above * pb, cudaMemcpyDeviceToDevice, s) !=
+                cudaSuccess)
+            fail(SP_E_CUDA, "loopback copy");
+        if (dn >= 0 && t.below > 0 &&
+            cudaMemcpyAsync(at(p, -t.below), at(h.prog[dn], nz - t.below), t.below * pb,
+                            cudaMemcpyDeviceToDevice, s) != cudaSuccess)
+            fail(SP_E_CUDA, "loopback copy");
+    }
+    if (cudaEventRecord(h.done[r], s) != cudaSuccess) fail(SP_E_CUDA, "event record");
+    h.barrier();
+    // my interior planes stay unmodified until the neighbours have pulled them
+    // (the send-completion of ncclSend)
+    for (int nb : {up, dn})
+        if (nb >= 0 && cudaStreamWaitEvent(s, h.done[nb], 0) != cudaSuccess)
+            fail(SP_E_CUDA, "stream wait");
+    h.barrier();  // no rank re-records its events before the others have waited on them
+}
+
+void exchange(stencil_program *p, const std::vector<Mode::Xfer> &x, void *stream) {
+    sp_comm *c = p->comm;
+    if (!c || c->nranks == 1 || x.empty()) return;
+    for (const Mode::Xfer &t : x)
+        if (!p->ptrs[t.arr]) fail(SP_E_STATE, "array '" + p->arrays[t.arr].name + "' is not bound");
+    if (c->hub) {
+        exchange_loopback(p, x, (cudaStream_t)stream);
+        return;
+    }
+    const int64_t plane = p->plane;
+    const int64_t nz = p->grid.nz_local;
+    const int64_t oz = p->layout.origin_z;
+    const ncclDataType_t dt = p->elem == 8 ? ncclFloat64 : ncclFloat32;
+    const int up = c->rank + 1 < c->nranks ? c->rank + 1 : -1;
+    const int dn = c->rank > 0 ? c->rank - 1 : -1;
+    ncclComm_t comm = (ncclComm_t)c->nccl;
+    cudaStream_t s = (cudaStream_t)stream;
+    nccl_check(ncclGroupStart(), "ncclGroupStart");
+    for (const Mode::Xfer &t : x) {
+        char *base = (char *)p->ptrs[t.arr];
+        auto at = [&](int64_t z) { return base + (z + oz) * plane * p->elem; };
+        // every rank runs the same schedule: the neighbour below receives `above`
+        // planes into its top ghost, the one above `below` planes into its bottom ghost
+        if (up >= 0) {
+            if (t.below > 0) nccl_check(ncclSend(at(nz - t.below), t.below * plane, dt, up, comm, s), "ncclSend");
+            if (t.above > 0) nccl_check(ncclRecv(at(nz), t.above * plane, dt, up, comm, s), "ncclRecv");
+        }
+        if (dn >= 0) {
+            if (t.above > 0) nccl_check(ncclSend(at(0), t.above * plane, dt, dn, comm, s), "ncclSend");
+            if (t.below > 0) nccl_check(ncclRecv(at(-t.below), t.below * plane, dt, dn, comm, s), "ncclRecv");
+        }
+    }
+    nccl_check(ncclGroupEnd(), "ncclGroupEnd");
+}
+
+}  // namespace sf
+
 void sf_comm_unique_id_impl(void *out) {
     ncclUniqueId id;
     nccl_check(ncclGetUniqueId(&id), "ncclGetUniqueId");
     static_assert(sizeof(ncclUniqueId) == 128, "ncclUniqueId size");
     std::memcpy(out, &id, 128);
+}
+
+static cudaStream_t new_stream() {
+    cudaStream_t s;
+    if (cudaStreamCreateWithFlags(&s, cudaStreamNonBlocking) != cudaSuccess)
+        sf::fail(SP_E_CUDA, "cudaStreamCreate (comm stream)");
+    return s;
 }
 
 sp_comm *sf_comm_create_impl(const void *idp, int32_t nranks, int32_t rank) {
@@ -35,11 +196,33 @@ sp_comm *sf_comm_create_impl(const void *idp, int32_t nranks, int32_t rank) {
     ncclComm_t comm;
     nccl_check(ncclCommInitRank(&comm, nranks, id, rank), "ncclCommInitRank");
     c->nccl = comm;
-    cudaStream_t s;
-    if (cudaStreamCreateWithFlags(&s, cudaStreamNonBlocking) != cudaSuccess)
-        sf::fail(SP_E_CUDA, "cudaStreamCreate (comm stream)");
-    c->comm_stream = s;
+    c->comm_stream = new_stream();
     return c.release();
+}
+
+void sf_comm_create_loopback_impl(int32_t nranks, sp_comm **out) {
+    sf::ensure_cuda();
+    auto hub = std::make_shared<sf::LoopHub>();
+    hub->n = nranks;
+    hub->prog.assign(nranks, nullptr);
+    for (int r = 0; r < nranks; ++r)
+        for (auto *v : {&hub->ready, &hub->done}) {
+            cudaEvent_t e;
+            if (cudaEventCreateWithFlags(&e, cudaEventDisableTiming) != cudaSuccess)
+                sf::fail(SP_E_CUDA, "cudaEventCreate");
+            v->push_back(e);
+        }
+    std::vector<std::unique_ptr<sp_comm>> cs;
+    for (int r = 0; r < nranks; ++r) {
+        std::unique_ptr<sp_comm> c(new sp_comm());
+        c->nranks = nranks;
+        c->rank = r;
+        cudaGetDevice(&c->device);
+        c->comm_stream = new_stream();
+        c->hub = hub;
+        cs.push_back(std::move(c));
+    }
+    for (int r = 0; r < nranks; ++r) out[r] = cs[r].release();
 }
 
 void sf_comm_destroy_impl(sp_comm *c) {
@@ -47,38 +230,3 @@ void sf_comm_destroy_impl(sp_comm *c) {
     if (c->comm_stream) cudaStreamDestroy((cudaStream_t)c->comm_stream);
     delete c;
 }
-
-namespace sf {
-
-void exchange(stencil_program *p, const std::vector<int> &arrays, int depth, void *stream) {
-    sp_comm *c = p->comm;
-    if (!c || c->nranks == 1 || arrays.empty()) return;
-    for (int a : arrays)
-        if (!p->ptrs[a]) fail(SP_E_STATE, "array '" + p->arrays[a].name + "' is not bound");
-    const int64_t plane = p->plane;
-    const int64_t nz = p->grid.nz_local;
-    const int64_t oz = p->layout.origin_z;
-    const size_t count = (size_t)(depth * plane);
-    const ncclDataType_t dt = p->elem == 8 ? ncclFloat64 : ncclFloat32;
-    const int up = c->rank + 1 < c->nranks ? c->rank + 1 : -1;
-    const int dn = c->rank > 0 ? c->rank - 1 : -1;
-    ncclComm_t comm = (ncclComm_t)c->nccl;
-    cudaStream_t s = (cudaStream_t)stream;
-    nccl_check(ncclGroupStart(), "ncclGroupStart");
-    for (int a : arrays) {
-        char *base = (char *)p->ptrs[a];
-        auto at = [&](int64_t z) { return base + (z + oz) * plane * p->elem; };
-        if (up >= 0) {
-            // my top `depth` interior planes -> up's bottom ghosts; up's bottom planes -> my top ghosts
-            nccl_check(ncclSend(at(nz - depth), count, dt, up, comm, s), "ncclSend");
-            nccl_check(ncclRecv(at(nz), count, dt, up, comm, s), "ncclRecv");
-        }
-        if (dn >= 0) {
-            nccl_check(ncclSend(at(0), count, dt, dn, comm, s), "ncclSend");
-            nccl_check(ncclRecv(at(-depth), count, dt, dn, comm, s), "ncclRecv");
-        }
-    }
-    nccl_check(ncclGroupEnd(), "ncclGroupEnd");
-}
-
-}  // namespace sf

@@ -265,7 +265,7 @@ void launch(stencil_program *p, Mode &m, int i, void *stream, int chunk_first, i
     int32_t ints[4] = {chunk_first, chunk_step, z_base, z_end};
     std::memcpy(base + L.int_off, ints, 16);
     void *args[] = {base};
-    if (L.pdl) {
+    if (L.pdl && !p->no_pdl) {
         // programmatic dependent launch: the kernel's prologue may overlap the previous
         // launch on the stream; griddepcontrol.wait in the kernel orders its data accesses
         CUlaunchAttribute attr[1];

@@ -131,14 +131,20 @@ struct Mode {
     struct alignas(64) Blk { unsigned char b[64]; };
     std::vector<std::vector<Blk>> params;  // per launch: tensor maps + pointers + ints
     std::vector<int> wave_off;  // z-wave schedule: plane offset (skew) per launch
+    // multi-rank halo exchange schedule: per launch, the ghost planes to receive first
+    struct Xfer { int arr, below, above; };
+    std::vector<std::vector<Xfer>> xsched;
+    bool xsched_ok = false;
 };
 
 }  // namespace sf
 
+namespace sf { struct LoopHub; }
 struct sp_comm_s {
-    void *nccl = nullptr;  // ncclComm_t
+    void *nccl = nullptr;  // ncclComm_t (null for a loopback communicator)
     int nranks = 1, rank = 0, device = 0;
     void *comm_stream = nullptr;  // cudaStream_t used for exchanges
+    std::shared_ptr<sf::LoopHub> hub;  // in-process virtual ranks (test transport)
 };
 
 struct stencil_program_s {
@@ -160,6 +166,7 @@ struct stencil_program_s {
     std::vector<std::vector<int>> plan_groups;  // gids per group
     int num_sms = 148;
     std::vector<void *> events;  // cudaEvent_t pool for exchange overlap
+    bool no_pdl = false;         // multi-rank schedule: plain stream order between launches
     std::vector<void *> wave_streams, wave_events;  // z-wave schedule: streams, events
     std::map<int, sp_tile_config> tune_fused, tune_unfused;  // sp_plan_tune overrides
 };
@@ -197,5 +204,8 @@ void ensure_cuda();
 void unload_mode(Mode &m);
 
 // comm.cpp
-void exchange(stencil_program *p, const std::vector<int> &arrays, int depth, void *stream);
+// receive `below` planes into the bottom ghost and `above` planes into the top
+// ghost of each array (the neighbours send the matching interior planes)
+void exchange(stencil_program *p, const std::vector<Mode::Xfer> &x, void *stream);
+void exchange_schedule(const stencil_program *p, Mode &m);
 }  // namespace sf

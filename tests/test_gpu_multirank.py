@@ -2,7 +2,7 @@
 
 Each rank is a Program over its slab (nz_global, z_offset, deep halo zhalo) with no
 communicator; before every fused group the test moves the ghost planes the library's
-exchange schedule names (sp_plan_exchange: arrays + depth) between the slab tensors
+exchange schedule names (sp_plan_exchange: arrays, planes below/above) between the slab tensors
 with device-to-device copies — exactly the planes run_fused would ncclSend/ncclRecv.
 The P-rank result must equal the single-domain result bit for bit: initialisation is
 a function of global coordinates and the fused kernels recompute intermediates on
@@ -90,13 +90,14 @@ def test_virtual_ranks_bitexact(cuda_device, cfg, ranks, fmad):
         fill(s, loc, dev, r * nzl, zhalo, nz_global=nzl * ranks)
         slabs.append(s)
     for i in range(slabs[0].n_launches("fused")):
-        names, depth = slabs[0].exchange_plan("fused", i)
-        assert depth <= zhalo
-        for r in range(ranks - 1):  # r <-> r+1
-            lo, hi = slabs[r], slabs[r + 1]
-            for n in names:
-                plane(hi, hi.tensors[n], -depth, depth).copy_(plane(lo, lo.tensors[n], nzl - depth, depth))
-                plane(lo, lo.tensors[n], nzl, depth).copy_(plane(hi, hi.tensors[n], 0, depth))
+        for n, below, above in slabs[0].exchange_plan("fused", i):
+            assert below <= zhalo and above <= zhalo
+            for r in range(ranks - 1):  # r <-> r+1
+                lo, hi = slabs[r], slabs[r + 1]
+                if below:
+                    plane(hi, hi.tensors[n], -below, below).copy_(plane(lo, lo.tensors[n], nzl - below, below))
+                if above:
+                    plane(lo, lo.tensors[n], nzl, above).copy_(plane(hi, hi.tensors[n], 0, above))
         for s in slabs:
             s.run_launch("fused", i)
     torch.cuda.synchronize()
@@ -105,3 +106,69 @@ def test_virtual_ranks_bitexact(cuda_device, cfg, ranks, fmad):
         want = single.interior_view(single.tensors[n])
         got = torch.cat([s.interior_view(s.tensors[n]) for s in slabs], dim=0)
         assert torch.equal(got, want), f"{cfg} {n}: slab result differs from single domain"
+
+
+@pytest.mark.parametrize("cfg,ranks,mode", [("C2", 2, "fused"), ("C5", 3, "fused"), ("C3", 2, "fused"),
+                                            ("C4", 2, "fused"), ("C4", 3, "unfused"),
+                                            ("chain3", 3, "fused"), ("C2box", 2, "fused"),
+                                            ("C2", 3, "unfused")])
+def test_loopback_ranks_run_bitexact(cuda_device, cfg, ranks, mode):
+    """The executor's own multi-rank path (run_fused / run_unfused with a communicator:
+    exchange schedule, interior planes overlapped with the exchange on the comm stream,
+    boundary planes after its event, no PDL) on in-process virtual ranks, one host
+    thread and one stream each; the loopback transport stands in for ncclSend/ncclRecv.
+    Two steps; the result must equal the single-domain result bit for bit (P9)."""
+    import threading
+    import torch
+    from paper_conf_hpdc_wahibm15_b200 import Comm, Program
+    nzl = 12
+    mk = {"C2": lambda nz: P.c2(nx=40, ny=24, nz=nz), "C5": lambda nz: P.c5(nx=32, ny=16, nz=nz),
+          "C3": lambda nz: P.c3(nx=48, ny=20, nz=nz), "C4": c4_small,
+          "chain3": lambda nz: P.resize(P.chain3(), 20, 12, nz), "C2box": c2_boxed}[cfg]
+    glob = mk(nzl * ranks)
+    plan = glob["plans"]["fused"]
+    dev = cuda_device
+    single = Program(glob)
+    single.set_plan(plan)
+    single.allocate(dev)
+    fill(single, glob, dev, 0, glob["grid"]["ghost"][2])
+    single.run(mode)
+    single.run(mode)
+    loc = mk(nzl)
+    probe = Program(loc, nz_global=nzl * ranks)
+    probe.set_plan(plan)
+    zhalo = max([max(r["z_below"], r["z_above"]) for m in ("fused", "unfused")
+                 for r in probe.reports(m)] + [loc["grid"]["ghost"][2]])
+    comms = Comm.loopback(ranks)
+    slabs = []
+    for r in range(ranks):
+        s = Program(loc, comm=comms[r], nz_global=nzl * ranks, z_offset=r * nzl, zhalo=zhalo)
+        s.set_plan(plan)
+        s.allocate(dev)
+        fill(s, loc, dev, r * nzl, zhalo, nz_global=nzl * ranks)
+        s.compile(mode)
+        slabs.append(s)
+    torch.cuda.synchronize()
+    errs = []
+
+    def drive(r):
+        try:
+            st = torch.cuda.Stream(device=dev)
+            for _ in range(2):
+                slabs[r].run(mode, st)
+            st.synchronize()
+        except Exception as e:  # surfaced below
+            errs.append(e)
+
+    th = [threading.Thread(target=drive, args=(r,)) for r in range(ranks)]
+    for t in th:
+        t.start()
+    for t in th:
+        t.join()
+    assert not errs, errs
+    torch.cuda.synchronize()
+    outs = [a["name"] for a in glob["arrays"] if a["role"] in ("out", "inout")]
+    for n in outs:
+        want = single.interior_view(single.tensors[n])
+        got = torch.cat([s.interior_view(s.tensors[n]) for s in slabs], dim=0)
+        assert torch.equal(got, want), f"{cfg} {n}: loopback multi-rank result differs from single domain"

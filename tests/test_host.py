@@ -272,12 +272,43 @@ def test_exchange_schedule_matches_reach():
     prog = P.c3(n=32)
     p = Program(prog, nz_global=64, z_offset=0, zhalo=5)
     p.set_plan(prog["plans"]["fission_fused"])
-    names, depth = p.exchange_plan("fused", 0)
-    assert names == ["A"] and depth == 5          # 7pt, 7pt, 13pt, 7pt chain: reach 1+1+2+1
-    names, depth = p.exchange_plan("fused", 1)
-    assert names == ["B"] and depth == 5          # O1 is read point-wise: no exchange
-    u_names, u_depth = p.exchange_plan("unfused", 2)
-    assert u_names == ["P1"] and u_depth == 2     # the 13-point kernel alone
+    assert p.exchange_plan("fused", 0) == [("A", 5, 5)]   # 7pt, 7pt, 13pt, 7pt chain: 1+1+2+1
+    assert p.exchange_plan("fused", 1) == [("B", 5, 5)]   # O1 is read point-wise: no exchange
+    # unfused: each array once per epoch (after its writer), before its first halo reader
+    want = {0: [("A", 1, 1), ("B", 1, 1)], 1: [("P", 1, 1)], 2: [("P1", 2, 2)], 3: [("P2", 1, 1)],
+            4: [("Q", 1, 1)], 5: [("Q1", 2, 2)], 6: [("Q2", 1, 1)], 7: []}
+    assert {i: p.exchange_plan("unfused", i) for i in range(8)} == want
+
+
+def test_exchange_schedule_hoists_unchanged_arrays():
+    """An array read beyond the slab by several launches between two writes is received
+    once, before the first of them, at the largest depth any of them needs (C4)."""
+    from synth.scale_les import c4
+    prog = c4(nx=64, ny=32, nz=32)
+    p = Program(prog, nz_global=64, z_offset=0, zhalo=4)
+    names = [a["name"] for a in prog["arrays"]]
+    n = p.n_launches("unfused")
+    got = {i: p.exchange_plan("unfused", i) for i in range(n)}
+    # replay: every halo read of every launch is covered by the last reception of that
+    # array since its last store, and nothing is received twice inside one epoch
+    fresh = {}
+    for i in range(n):
+        for a, lo, hi in got[i]:
+            assert a not in fresh, f"{a} received twice in one epoch"
+            fresh[a] = (lo, hi)
+        r = p.report("unfused", i)
+        k = prog["kernels"][i]
+        for st in k["stmts"]:
+            for t in st["terms"]:
+                for tap in ([t["a"]] + ([t["b"]] if t.get("b") else [])):
+                    arr, dz = tap[0], tap[3]
+                    if dz:
+                        lo, hi = fresh[arr]
+                        assert (-dz <= lo) if dz < 0 else (dz <= hi), (i, arr, dz)
+        for st in k["stmts"]:
+            fresh.pop(st["out"], None)
+    assert sum(len(v) for v in got.values()) < sum(
+        1 for k in prog["kernels"] for st in k["stmts"] for t in st["terms"])
 
 
 def test_deep_halo_must_cover_reach():

@@ -93,23 +93,26 @@ def _worker(rank, world, port, cfg, q, shrink=0):
             return a[hz + p0:hz + p0 + n]
 
         for gi in range(len(plan)):
-            xnames, depth = prog.exchange_plan("fused", gi)
-            depth -= shrink
+            xs = prog.exchange_plan("fused", gi)
             reqs = []
-            for n in (xnames if depth > 0 else []):
+            dt = torch.float64 if loc["dtype"] == "f64" else torch.float32
+            for n, below, above in xs:
+                below, above = max(0, below - shrink), max(0, above - shrink)
                 a = arrs[n]
-                if rank + 1 < world:   # my top interior planes -> up; up's bottom -> my top ghosts
-                    send = torch.from_numpy(planes(a, D + nzl - depth, depth).copy())
-                    dist.send(send, dst=rank + 1)
-                    recv = torch.empty_like(send)
-                    dist.recv(recv, src=rank + 1)
-                    planes(a, D + nzl, depth)[...] = recv.numpy()
+                if rank + 1 < world:   # my top `below` planes -> up's bottom ghost; up's bottom -> my top
+                    if below:
+                        dist.send(torch.from_numpy(planes(a, D + nzl - below, below).copy()), dst=rank + 1)
+                    if above:
+                        recv = torch.empty(planes(a, 0, above).shape, dtype=dt)
+                        dist.recv(recv, src=rank + 1)
+                        planes(a, D + nzl, above)[...] = recv.numpy()
                 if rank > 0:
-                    recv = torch.empty(planes(a, 0, depth).shape, dtype=torch.float64 if loc["dtype"] == "f64" else torch.float32)
-                    dist.recv(recv, src=rank - 1)
-                    planes(a, D - depth, depth)[...] = recv.numpy()
-                    send = torch.from_numpy(planes(a, D, depth).copy())
-                    dist.send(send, dst=rank - 1)
+                    if below:
+                        recv = torch.empty(planes(a, 0, below).shape, dtype=dt)
+                        dist.recv(recv, src=rank - 1)
+                        planes(a, D - below, below)[...] = recv.numpy()
+                    if above:
+                        dist.send(torch.from_numpy(planes(a, D, above).copy()), dst=rank - 1)
             del reqs
             box = (0, ext[0], 0, ext[1], box_k[0], box_k[1])
             sub_programs[gi].run(arrs, box=box, n=ext)
@@ -117,7 +120,7 @@ def _worker(rank, world, port, cfg, q, shrink=0):
                 for n, a in arrs.items():
                     own = a[hz + D:hz + D + nzl]
                     if np.isnan(own).any():
-                        print(f"rank {rank} after group {gi} exchange {xnames}@{depth}: {n} own NaN planes "
+                        print(f"rank {rank} after group {gi} exchange {xs}: {n} own NaN planes "
                               f"{sorted(set(np.argwhere(np.isnan(own))[:, 0].tolist()))}", flush=True)
         outs = [a["name"] for a in loc["arrays"] if a["role"] in ("out", "inout")]
         mine = {n: arrs[n][hz + D:hz + D + nzl, hy:hy + ext[1], hx:hx + ext[0]].copy() for n in outs}

@@ -131,8 +131,7 @@ static void run_waves(stencil_program *p, Mode &m, void *stream) {
     auto go = [&](int w, int i, void *s) {
         int z0, z1;
         if (m.launches[i].dead || !range(w, i, &z0, &z1)) return false;
-        const int zc = m.launches[i].zc;
-        launch(p, m, i, s, 0, 1, (z1 - z0 + zc - 1) / zc, z0, z1);
+        launch(p, m, i, s, z0, z1);
         return true;
     };
     if (ns == 1) {
@@ -191,7 +190,7 @@ static void run_mode(stencil_program *p, int mode, void *stream) {
         return;
     }
     if (!multi) {
-        for (size_t i = 0; i < m.launches.size(); ++i) launch(p, m, (int)i, stream, 0, 1, m.launches[i].nch);
+        for (size_t i = 0; i < m.launches.size(); ++i) launch(p, m, (int)i, stream);
         return;
     }
     // several ranks: programmatic dependent launch is not used across the exchange's
@@ -209,9 +208,8 @@ static void run_mode(stencil_program *p, int mode, void *stream) {
         p->events.push_back(ev);
     }
     cudaEvent_t ready = (cudaEvent_t)p->events[0], done = (cudaEvent_t)p->events[1];
-    auto planes = [&](int i, int z0, int z1) {
-        const int zc = m.launches[i].zc;
-        if (z1 > z0) launch(p, m, i, stream, 0, 1, (z1 - z0 + zc - 1) / zc, z0, z1);
+    auto planes = [&](int i, int z0, int z1, int z2 = 0, int z3 = 0) {
+        launch(p, m, i, stream, z0, z1, z2, z3);
     };
     for (size_t i = 0; i < m.launches.size(); ++i) {
         Launch &L = m.launches[i];
@@ -234,8 +232,7 @@ static void run_mode(stencil_program *p, int mode, void *stream) {
         if (cudaStreamWaitEvent((cudaStream_t)stream, done, 0) != cudaSuccess)
             fail(SP_E_CUDA, "stream wait");
         if (split) {
-            planes((int)i, 0, zb);
-            planes((int)i, ze, nz);
+            planes((int)i, 0, zb, ze, nz);  // both boundary ranges in one launch
         } else {
             planes((int)i, 0, nz);
         }
@@ -527,7 +524,7 @@ sp_status sp_run_launch(stencil_program *p, int32_t mode, int32_t i, sp_stream s
         Mode &m = mode_of(p, mode);
         if (i < 0 || i >= (int)m.launches.size()) fail(SP_E_ARG, "launch index out of range");
         load_mode(p, m);
-        launch(p, m, i, stream, 0, 1, m.launches[i].nch);
+        launch(p, m, i, stream);
     });
 }
 

@@ -178,7 +178,7 @@ std::string generate_launch(const stencil_program *p, Launch &L, int index, bool
     const int narr = (int)L.slot_arr.size();
     L.ptr_off = 128 * (size_t)std::max(nin, 1);
     L.int_off = L.ptr_off + 8 * (size_t)std::max(narr, 1);
-    L.param_size = (L.int_off + 16 + 63) / 64 * 64;
+    L.param_size = (L.int_off + 24 + 63) / 64 * 64;
     const int NB = L.nbar_full, NE = L.nbar_empty;
 
     o << "// generated by stencilfuse codegen: " << (fused ? "fused group " : "original kernel ")
@@ -197,7 +197,7 @@ std::string generate_launch(const stencil_program *p, Launch &L, int index, bool
     o << "constexpr int OXA = " << lay.origin_x << ", OYA = " << lay.origin_y
       << ", OZA = " << lay.origin_z << ";\n";
     o << "struct __align__(64) Params { SfTmap tm[" << std::max(nin, 1) << "]; T *arr["
-      << std::max(narr, 1) << "]; int chunk_first, chunk_step, z_base, z_end; };\n";
+      << std::max(narr, 1) << "]; int n_lo, z_mid, z_hi, z_base, z_end, pad_; };\n";
     o << "static_assert(sizeof(SfTmap) * " << std::max(nin, 1) << " == " << L.ptr_off
       << ", \"param layout\");\n";
     // statement coefficients live in constant memory: FP64 FMA/MUL take them as
@@ -220,9 +220,11 @@ std::string generate_launch(const stencil_program *p, Launch &L, int index, bool
     o << "  using namespace " << L.fn << "_ns;\n";
     o << "  extern __shared__ __align__(128) unsigned char sf_smem[];\n";
     o << "  const int tid = threadIdx.x;\n";
-    o << "  const int chunk = p.chunk_first + (int)blockIdx.z * p.chunk_step;\n";
-    o << "  const int X0 = (int)blockIdx.x * TX, Y0 = (int)blockIdx.y * TY, Z0 = p.z_base + chunk * ZC;\n";
-    o << "  const int zc = min(ZC, p.z_end - Z0);\n";
+    // chunks [0, n_lo) tile planes [z_base, z_mid), the others [z_hi, z_end)
+    o << "  const int bz = (int)blockIdx.z, lo = bz < p.n_lo;\n";
+    o << "  const int X0 = (int)blockIdx.x * TX, Y0 = (int)blockIdx.y * TY,\n"
+         "            Z0 = lo ? p.z_base + bz * ZC : p.z_hi + (bz - p.n_lo) * ZC;\n";
+    o << "  const int zc = min(ZC, (lo ? p.z_mid : p.z_end) - Z0);\n";
     o << "  sf_u64 *full = (sf_u64 *)(sf_smem + " << L.bar_off << ");\n";
     if (tma) o << "  sf_u64 *empty = full + " << NB << ";\n";
     for (int a = 0; a < nin; ++a) {

@@ -17,7 +17,8 @@
 
 #include <algorithm>
 #include <chrono>
-#include <condition_variable>
+#include <atomic>
+#include <thread>
 #include <cstring>
 
 #include "sf_internal.h"
@@ -31,27 +32,27 @@ namespace sf {
 
 struct LoopHub {
     int n = 0;
-    std::mutex mu;
-    std::condition_variable cv;
-    int arrived = 0;
-    uint64_t gen = 0;
+    std::atomic<int> arrived{0};
+    std::atomic<uint64_t> gen{0};
     std::vector<stencil_program *> prog;
     std::vector<cudaEvent_t> ready, done;
 
-    // all n virtual ranks meet; a missing rank (an error on its thread) times out
+    // all n virtual ranks meet (spinning: the exchange issues device work between
+    // barriers and a sleeping wake-up would starve the GPU); a missing rank (an
+    // error on its thread) times out
     void barrier() {
-        std::unique_lock<std::mutex> lk(mu);
-        const uint64_t g = gen;
-        if (++arrived == n) {
-            arrived = 0;
-            ++gen;
-            cv.notify_all();
+        const uint64_t g = gen.load(std::memory_order_acquire);
+        if (arrived.fetch_add(1, std::memory_order_acq_rel) + 1 == n) {
+            arrived.store(0, std::memory_order_relaxed);
+            gen.fetch_add(1, std::memory_order_acq_rel);
             return;
         }
-        if (!cv.wait_for(lk, std::chrono::seconds(120), [&] { return gen != g; })) {
-            --arrived;
-            fail(SP_E_STATE, "loopback exchange: a virtual rank did not reach the exchange "
-                             "(each rank must run the same plan on its own host thread)");
+        const auto t0 = std::chrono::steady_clock::now();
+        for (uint64_t k = 1; gen.load(std::memory_order_acquire) == g; ++k) {
+            if (k % 64 == 0) std::this_thread::yield();
+            if (k % 4096 == 0 && std::chrono::steady_clock::now() - t0 > std::chrono::seconds(120))
+                fail(SP_E_STATE, "loopback exchange: a virtual rank did not reach the exchange "
+                                 "(each rank must run the same plan on its own host thread)");
         }
     }
     ~LoopHub() {

@@ -255,15 +255,23 @@ static void build_params(stencil_program *p, Mode &m) {
     m.maps_version = p->bind_version;
 }
 
-void launch(stencil_program *p, Mode &m, int i, void *stream, int chunk_first, int chunk_step,
-            int nchunks, int z_base, int z_end) {
+void launch(stencil_program *p, Mode &m, int i, void *stream, int z0, int z1, int z2, int z3) {
     Launch &L = m.launches[i];
-    if (L.dead || nchunks <= 0) return;
+    if (L.dead || L.zc <= 0) return;
+    const int nz = (int)p->grid.nz_local;
+    if (z1 < 0) z1 = nz;
+    z0 = std::max(0, z0);
+    z1 = std::min(nz, z1);
+    z2 = std::max(z2, z1);
+    z3 = std::min(z3, nz);
+    const int n_lo = z1 > z0 ? (z1 - z0 + L.zc - 1) / L.zc : 0;
+    const int n_hi = z3 > z2 ? (z3 - z2 + L.zc - 1) / L.zc : 0;
+    const int nchunks = n_lo + n_hi;
+    if (nchunks <= 0) return;
     build_params(p, m);
     unsigned char *base = m.params[i][0].b;
-    if (z_end < 0) z_end = (int)p->grid.nz_local;
-    int32_t ints[4] = {chunk_first, chunk_step, z_base, z_end};
-    std::memcpy(base + L.int_off, ints, 16);
+    int32_t ints[6] = {n_lo, z1, z2, z0, z3, 0};
+    std::memcpy(base + L.int_off, ints, 24);
     void *args[] = {base};
     if (L.pdl && !p->no_pdl) {
         // programmatic dependent launch: the kernel's prologue may overlap the previous

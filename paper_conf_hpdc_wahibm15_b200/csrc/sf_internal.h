@@ -196,10 +196,10 @@ double codegen_smem_loads(const Launch &L);  // shared-memory loads per core poi
 // jit.cpp
 void compile_mode(stencil_program *p, Mode &m);
 void load_mode(stencil_program *p, Mode &m);
-// chunks chunk_first + c*chunk_step (c < nchunks) of the z range [z_base, z_end)
-// (z_end < 0: the whole local slab); chunk c starts at plane z_base + chunk*zc
-void launch(stencil_program *p, Mode &m, int i, void *stream, int chunk_first, int chunk_step,
-            int nchunks, int z_base = 0, int z_end = -1);
+// one launch over output planes [z0, z1) and [z2, z3) of the slab (z1 < 0: the
+// whole slab; an empty second range by default), each tiled by chunks of zc planes
+void launch(stencil_program *p, Mode &m, int i, void *stream, int z0 = 0, int z1 = -1, int z2 = 0,
+            int z3 = 0);
 void ensure_cuda();
 void unload_mode(Mode &m);
 

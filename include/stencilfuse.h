@@ -166,6 +166,35 @@ sp_status sp_comm_create(const void *nccl_unique_id, int32_t nranks, int32_t ran
  * interior/boundary planes, events) is the NCCL path's.  Destroy each with
  * sp_comm_destroy. */
 sp_status sp_comm_create_loopback(int32_t nranks, sp_comm **out);
+
+/* ---- peer-push halo exchange (option "xpush" = 1, several ranks) ----------
+ * SURVEY.md §8(e) "B200-native step beyond send/recv" / §8(f) NEXT #2.  With
+ * the option set, an epoch of a TEMP array that begins at a store (see
+ * sp_plan_exchange) is not exchanged by the communicator: the storing kernel
+ * writes the bottom/top planes the neighbours' readers need straight into the
+ * neighbours' ghost planes (st.global to peer memory over NVLink/NVSwitch), and
+ * every kernel of the rank runs a progress protocol with its neighbours: chunks
+ * within reach of a slab end wait (in the kernel) until both neighbours have
+ * completed the previous launch, and the last CTA of each kernel publishes its
+ * completion to both neighbours (fence.sc.sys + st.release.sys).  Step-start
+ * epochs (IN arrays, previous-step state) still travel through the communicator.
+ * Every rank must bind, before its first run:
+ *   - sp_bind_peer(array, side, ptr) for each TEMP array: the neighbour's buffer
+ *     of that array (side 0 = rank-1, 1 = rank+1) mapped in this process;
+ *   - sp_bind_peer_signal(side, ptr): the neighbour's signal block
+ *     (sp_signal_buffer on that rank, 64 B of device memory it owns).
+ * Unbound neighbours of an existing side give SP_E_STATE at the run.  A rank
+ * that stops running makes its neighbours' waiting kernels trap after 20 s
+ * (no hang).  Layouts must be identical on all ranks (same grid and zhalo). */
+sp_status sp_signal_buffer(stencil_program *prog, void **out);
+sp_status sp_bind_peer(stencil_program *prog, int32_t array, int32_t side, void *peer_ptr);
+sp_status sp_bind_peer_signal(stencil_program *prog, int32_t side, void *peer_signal);
+/* CUDA IPC of a device pointer (any pointer inside a cudaMalloc allocation, e.g.
+ * a torch tensor): 64-byte handle of the allocation + the pointer's offset in it.
+ * sp_ipc_open maps it in another process (once per allocation; mappings live
+ * until the process exits).  SP_E_CUDA on failure. */
+sp_status sp_ipc_export(const void *dev_ptr, void *handle64, int64_t *offset);
+sp_status sp_ipc_open(const void *handle64, int64_t offset, void **dev_ptr);
 void sp_comm_destroy(sp_comm *comm);
 
 /* ---- program ------------------------------------------------------------ */
@@ -280,6 +309,11 @@ sp_status sp_plan_exchange(stencil_program *prog, int32_t mode, int32_t launch, 
 sp_status sp_plan_wave_offsets(stencil_program *prog, int32_t cap, int32_t *off, int32_t *n);
 /* JIT-compile (NVRTC, sm_100a) without launching; needs no GPU. */
 sp_status sp_compile(stencil_program *prog, int32_t mode);
+/* Compile if needed and load the mode's modules on the current device (needs a
+ * GPU).  run_* load lazily; call this first when ranks are driven from several
+ * threads of one process (loopback), since a module load may synchronise the
+ * device while a neighbour's kernels wait for this rank. */
+sp_status sp_load(stencil_program *prog, int32_t mode);
 
 /* ---- execution ---------------------------------------------------------- */
 /* Every original kernel once, in program order: one launch per kernel, each

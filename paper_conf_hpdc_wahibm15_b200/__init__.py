@@ -195,6 +195,59 @@ class Program:
         _check(lib().stencil_program_bind(self.handle, self.index[name],
                                           ctypes.c_void_p(tensor.data_ptr())))
 
+    # ---------------------------------------------------------- peer push (option xpush)
+    def temp_names(self):
+        return [a["name"] for a in self.prog["arrays"] if a["role"] == "temp"]
+
+    def signal_buffer(self):
+        """Device address of this program's 64-B signal block (sp_signal_buffer)."""
+        out = ctypes.c_void_p()
+        _check(lib().sp_signal_buffer(self.handle, ctypes.byref(out)))
+        return out.value
+
+    def bind_peer(self, name, side, ptr):
+        _check(lib().sp_bind_peer(self.handle, self.index[name], int(side), ctypes.c_void_p(ptr)))
+
+    def bind_peer_signal(self, side, ptr):
+        _check(lib().sp_bind_peer_signal(self.handle, int(side), ctypes.c_void_p(ptr)))
+
+    @staticmethod
+    def connect_peers_local(progs):
+        """Peer-push wiring of in-process ranks (loopback virtual ranks on one device):
+        each rank's neighbour buffers are the neighbours' own tensors."""
+        for r, p in enumerate(progs):
+            for side, q in ((0, r - 1), (1, r + 1)):
+                if 0 <= q < len(progs):
+                    for n in p.temp_names():
+                        p.bind_peer(n, side, progs[q].tensors[n].data_ptr())
+                    p.bind_peer_signal(side, progs[q].signal_buffer())
+
+    def connect_peers(self, rank, world, group=None):
+        """Peer-push wiring across processes: CUDA IPC handles of every TEMP array and
+        of the signal block, all-gathered over torch.distributed, opened for the two
+        z-neighbours (collective over the group)."""
+        import torch.distributed as dist
+        mine = {}
+        for n in self.temp_names() + ["__signal__"]:
+            ptr = self.signal_buffer() if n == "__signal__" else self.tensors[n].data_ptr()
+            h = (ctypes.c_ubyte * 64)()
+            off = ctypes.c_int64()
+            _check(lib().sp_ipc_export(ctypes.c_void_p(ptr), h, ctypes.byref(off)))
+            mine[n] = (bytes(h), off.value)
+        allv = [None] * world
+        dist.all_gather_object(allv, mine, group=group)
+        for side, q in ((0, rank - 1), (1, rank + 1)):
+            if not 0 <= q < world:
+                continue
+            for n, (h, off) in allv[q].items():
+                out = ctypes.c_void_p()
+                hb = (ctypes.c_ubyte * 64)(*h)
+                _check(lib().sp_ipc_open(hb, off, ctypes.byref(out)))
+                if n == "__signal__":
+                    self.bind_peer_signal(side, out.value)
+                else:
+                    self.bind_peer(n, side, out.value)
+
     def padded_view(self, tensor, hz=None):
         """View of the dense padded region [nz+2hz][ny+2hy][nx+2hx] (ghost width per side)."""
         L = self.layout
@@ -306,6 +359,10 @@ class Program:
         buf = (ctypes.c_int32 * max(1, n.value))()
         _check(lib().sp_plan_wave_offsets(self.handle, n.value, buf, ctypes.byref(n)))
         return [buf[j] for j in range(n.value)]
+
+    def load(self, mode):
+        """Compile if needed and load the mode's kernels on the current device (sp_load)."""
+        _check(lib().sp_load(self.handle, self._mode(mode)))
 
     def compile(self, mode):
         _check(lib().sp_compile(self.handle, self._mode(mode)))

@@ -81,11 +81,12 @@ class SpGroupReport(ctypes.Structure):
 
 # every symbol include/stencilfuse.h declares (checked by tests/test_abi.py)
 EXPORTS = [
-    "sp_comm_unique_id", "sp_comm_create", "sp_comm_create_loopback", "sp_comm_destroy", "stencil_program_create",
+    "sp_comm_unique_id", "sp_comm_create", "sp_comm_create_loopback", "sp_comm_destroy",
+    "sp_signal_buffer", "sp_bind_peer", "sp_bind_peer_signal", "sp_ipc_export", "sp_ipc_open", "stencil_program_create",
     "stencil_program_destroy", "stencil_program_layout", "stencil_program_bind",
     "sp_program_set_option", "sp_program_counts", "sp_program_edges", "sp_fission_components",
     "fusion_plan_set", "sp_plan_greedy", "sp_plan_count", "sp_plan_report", "fusion_plan_report", "sp_plan_source",
-    "sp_plan_exchange", "sp_plan_wave_offsets", "sp_plan_tune", "sp_compile", "run_unfused", "run_fused", "sp_run_launch", "exchange_halos", "sp_last_error",
+    "sp_plan_exchange", "sp_plan_wave_offsets", "sp_plan_tune", "sp_compile", "sp_load", "run_unfused", "run_fused", "sp_run_launch", "exchange_halos", "sp_last_error",
 ]
 
 _lib = None
@@ -104,6 +105,11 @@ def lib():
             "sp_comm_unique_id": [vp],
             "sp_comm_create": [vp, i32, i32, P(vp)],
             "sp_comm_create_loopback": [i32, P(vp)],
+            "sp_signal_buffer": [vp, P(vp)],
+            "sp_bind_peer": [vp, i32, i32, vp],
+            "sp_bind_peer_signal": [vp, i32, vp],
+            "sp_ipc_export": [vp, vp, P(i64)],
+            "sp_ipc_open": [vp, i64, P(vp)],
             "stencil_program_create": [P(SpGrid), i32, P(SpArrayDesc), i32, P(SpKernel), vp, P(vp)],
             "stencil_program_layout": [vp, P(SpLayout)],
             "stencil_program_bind": [vp, i32, vp],
@@ -118,6 +124,7 @@ def lib():
             "fusion_plan_report": [vp, i32, P(SpGroupReport)],
             "sp_plan_source": [vp, i32, ctypes.c_char_p, ctypes.c_size_t, P(ctypes.c_size_t)],
             "sp_compile": [vp, i32],
+            "sp_load": [vp, i32],
             "sp_plan_exchange": [vp, i32, i32, i32, P(i32), P(i32), P(i32), P(i32)],
             "sp_plan_wave_offsets": [vp, i32, P(i32), P(i32)],
             "sp_plan_tune": [vp, i32, i32, P(SpTileConfig)],

@@ -20,6 +20,8 @@ sp_comm *sf_comm_create_impl(const void *, int32_t, int32_t);
 void sf_comm_destroy_impl(sp_comm *);
 void sf_comm_unique_id_impl(void *);
 void sf_comm_create_loopback_impl(int32_t, sp_comm **);
+void sf_ipc_export_impl(const void *, void *, int64_t *);
+void *sf_ipc_open_impl(const void *, int64_t);
 
 namespace sf {
 static thread_local std::string t_err;
@@ -200,7 +202,7 @@ static void run_mode(stencil_program *p, int mode, void *stream) {
     if (!m.xsched_ok) exchange_schedule(p, m);
     p->no_pdl = true;
     const int nz = (int)p->grid.nz_local;
-    cudaStream_t cs = (cudaStream_t)p->comm->comm_stream;
+    cudaStream_t cs = (cudaStream_t)comm_stream(p->comm);
     while (p->events.size() < 2) {
         cudaEvent_t ev;
         if (cudaEventCreateWithFlags(&ev, cudaEventDisableTiming) != cudaSuccess)
@@ -286,6 +288,7 @@ void stencil_program_destroy(stencil_program *p) {
         for (void *e : p->events) cudaEventDestroy((cudaEvent_t)e);
         for (void *e : p->wave_events) cudaEventDestroy((cudaEvent_t)e);
         for (void *s : p->wave_streams) cudaStreamDestroy((cudaStream_t)s);
+        if (p->sig) cudaFree(p->sig);
     });
     delete p;
 }
@@ -306,6 +309,47 @@ sp_status stencil_program_bind(stencil_program *p, int32_t array, void *dev_ptr)
             p->ptrs[array] = dev_ptr;
             p->bind_version++;
         }
+    });
+}
+
+sp_status sp_signal_buffer(stencil_program *p, void **out) {
+    return guard([&] {
+        if (!p || !out) fail(SP_E_ARG, "null argument");
+        *out = signal_block(p);
+    });
+}
+
+sp_status sp_bind_peer(stencil_program *p, int32_t array, int32_t side, void *peer_ptr) {
+    return guard([&] {
+        if (!p || array < 0 || array >= (int)p->arrays.size() || side < 0 || side > 1)
+            fail(SP_E_ARG, "bad array index or side");
+        if (peer_ptr && ((uintptr_t)peer_ptr & 255)) fail(SP_E_ARG, "peer pointer must be 256-byte aligned");
+        p->peer[array][side] = peer_ptr;
+        p->bind_version++;
+    });
+}
+
+sp_status sp_bind_peer_signal(stencil_program *p, int32_t side, void *peer_signal) {
+    return guard([&] {
+        if (!p || side < 0 || side > 1) fail(SP_E_ARG, "bad side");
+        p->peer_sig[side] = peer_signal;
+        p->bind_version++;
+    });
+}
+
+sp_status sp_ipc_export(const void *dev_ptr, void *handle64, int64_t *offset) {
+    return guard([&] {
+        if (!dev_ptr || !handle64 || !offset) fail(SP_E_ARG, "null argument");
+        ensure_cuda();
+        sf_ipc_export_impl(dev_ptr, handle64, offset);
+    });
+}
+
+sp_status sp_ipc_open(const void *handle64, int64_t offset, void **dev_ptr) {
+    return guard([&] {
+        if (!handle64 || !dev_ptr || offset < 0) fail(SP_E_ARG, "bad argument");
+        ensure_cuda();
+        *dev_ptr = sf_ipc_open_impl(handle64, offset);
     });
 }
 
@@ -334,6 +378,7 @@ sp_status sp_program_set_option(stencil_program *p, const char *key, int64_t v) 
         else if (k == "factor") o.factor = v != 0;
         else if (k == "zwave") o.zwave = (int)v;
         else if (k == "zwave_streams") o.zwave_streams = std::max(1, std::min(8, (int)v));
+        else if (k == "xpush") o.xpush = (int)std::min<int64_t>(v, 2);
         else if (k == "l2_flush") {}
         else fail(SP_E_ARG, "unknown option '" + k + "'");
         if (v < 0 && k != "prefetch") fail(SP_E_ARG, "negative option value");
@@ -504,6 +549,13 @@ sp_status sp_compile(stencil_program *p, int32_t mode) {
     });
 }
 
+sp_status sp_load(stencil_program *p, int32_t mode) {
+    return guard([&] {
+        if (!p) fail(SP_E_ARG, "null program");
+        load_mode(p, mode_of(p, mode));
+    });
+}
+
 sp_status run_unfused(stencil_program *p, sp_stream stream) {
     return guard([&] {
         if (!p) fail(SP_E_ARG, "null program");
@@ -524,6 +576,7 @@ sp_status sp_run_launch(stencil_program *p, int32_t mode, int32_t i, sp_stream s
         Mode &m = mode_of(p, mode);
         if (i < 0 || i >= (int)m.launches.size()) fail(SP_E_ARG, "launch index out of range");
         load_mode(p, m);
+        if (p->comm && p->comm->nranks > 1) p->no_pdl = true;
         launch(p, m, i, stream);
     });
 }

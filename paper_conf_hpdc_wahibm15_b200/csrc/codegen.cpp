@@ -178,7 +178,9 @@ std::string generate_launch(const stencil_program *p, Launch &L, int index, bool
     const int narr = (int)L.slot_arr.size();
     L.ptr_off = 128 * (size_t)std::max(nin, 1);
     L.int_off = L.ptr_off + 8 * (size_t)std::max(narr, 1);
-    L.param_size = (L.int_off + 24 + 63) / 64 * 64;
+    L.xp_off = L.int_off + 24;
+    const int NPU = (int)L.pushes.size();
+    L.param_size = (L.xp_off + (L.xp ? 40 + 16 * (size_t)std::max(NPU, 1) : 0) + 63) / 64 * 64;
     const int NB = L.nbar_full, NE = L.nbar_empty;
 
     o << "// generated by stencilfuse codegen: " << (fused ? "fused group " : "original kernel ")
@@ -197,7 +199,11 @@ std::string generate_launch(const stencil_program *p, Launch &L, int index, bool
     o << "constexpr int OXA = " << lay.origin_x << ", OYA = " << lay.origin_y
       << ", OZA = " << lay.origin_z << ";\n";
     o << "struct __align__(64) Params { SfTmap tm[" << std::max(nin, 1) << "]; T *arr["
-      << std::max(narr, 1) << "]; int n_lo, z_mid, z_hi, z_base, z_end, pad_; };\n";
+      << std::max(narr, 1) << "]; int n_lo, z_mid, z_hi, z_base, z_end, pad_;";
+    if (L.xp)  // peer-push protocol: own signal block, neighbours' blocks, peer buffers
+        o << "\n  unsigned long long *xs_self, *xs_own, *xs_dn, *xs_up; unsigned *xs_ctr; T *xp["
+          << std::max(NPU, 1) << "][2];";
+    o << " };\n";
     o << "static_assert(sizeof(SfTmap) * " << std::max(nin, 1) << " == " << L.ptr_off
       << ", \"param layout\");\n";
     // statement coefficients live in constant memory: FP64 FMA/MUL take them as
@@ -221,7 +227,10 @@ std::string generate_launch(const stencil_program *p, Launch &L, int index, bool
     o << "  extern __shared__ __align__(128) unsigned char sf_smem[];\n";
     o << "  const int tid = threadIdx.x;\n";
     // chunks [0, n_lo) tile planes [z_base, z_mid), the others [z_hi, z_end)
-    o << "  const int bz = (int)blockIdx.z, lo = bz < p.n_lo;\n";
+    if (L.xp)  // chunks next to the slab ends (which may wait for the neighbours) go last
+        o << "  const int bz = ((int)blockIdx.z + 1) % (int)gridDim.z, lo = bz < p.n_lo;\n";
+    else
+        o << "  const int bz = (int)blockIdx.z, lo = bz < p.n_lo;\n";
     o << "  const int X0 = (int)blockIdx.x * TX, Y0 = (int)blockIdx.y * TY,\n"
          "            Z0 = lo ? p.z_base + bz * ZC : p.z_hi + (bz - p.n_lo) * ZC;\n";
     o << "  const int zc = min(ZC, (lo ? p.z_mid : p.z_end) - Z0);\n";
@@ -300,6 +309,22 @@ std::string generate_launch(const stencil_program *p, Launch &L, int index, bool
         for (int a = 0; a < nin; ++a) o << "    sf_prefetch_tmap(&p.tm[" << a << "]);\n";
     }
     o << "  }\n  __syncthreads();\n";
+    if (L.xp) {
+        // peer-push protocol: this kernel is number seq of
+        // the rank's launches; a chunk within xp_dw planes of a slab end reads ghost
+        // planes the neighbours push, or pushes into theirs, so it first waits until
+        // both neighbours have completed launch seq-1 (RAW: their pushes are visible;
+        // WAR: they have finished reading the ghosts this launch overwrites)
+        o << "  sf_pdl_wait();\n";
+        o << "  const unsigned long long xs_seq = sf_ld_volatile_u64(p.xs_self) + 1;\n";
+        if (std::getenv("SF_DEBUG_XP"))
+            o << "  if (tid == 0) printf(\"[" << L.fn << "] own=%p seq=%llu Z0=%d zc=%d nlo=%d blk=%d,%d,%d\\n\", p.xs_own, xs_seq, Z0, zc, p.n_lo, blockIdx.x, blockIdx.y, blockIdx.z);\n";
+        if (L.xp_dw > 0) {
+            o << "  if (Z0 < " << L.xp_dw << " || Z0 + zc > NZ - " << L.xp_dw << ") {\n";
+            o << "    if (tid == 0) sf_xs_wait(p.xs_own, p.xs_dn != nullptr, p.xs_up != nullptr, xs_seq - 1);\n";
+            o << "    __syncthreads();\n  }\n";
+        }
+    }
     // PDL measured r1: -1.6 % on the fused C4 step, +37 % on the 40-launch unfused step
     // (dependent grids parked on griddepcontrol.wait): fused groups only unless pdl=2
     const bool pdl = fused ? p->opt.pdl >= 1 : p->opt.pdl >= 2;
@@ -786,36 +811,59 @@ std::string generate_launch(const stencil_program *p, Launch &L, int index, bool
                       << iy << "_" << jx << ";\n";
         }
         if (G.stored) {
+            // the tile's core points of this plane, stored at base pointer `gbn`
+            auto stores = [&](const std::string &gbn, const std::string &ind) {
+                o << ind << "if (fast) {\n";
+                for (int iy = 0; iy < VY; ++iy) {
+                    if (vec_ok) {
+                        for (int jx = 0; jx < VX; jx += VW) {
+                            o << ind << "  sf_st_v(" << gbn << " + (" << iy << " * XP + " << jx << "), T2{";
+                            for (int e2 = 0; e2 < VW; ++e2)
+                                o << (e2 ? ", " : "") << "o" << iy << "_" << jx + e2;
+                            o << "});\n";
+                        }
+                    } else {
+                        for (int jx = 0; jx < VX; ++jx)
+                            o << ind << "  sf_st(" << gbn << " + (" << iy << " * XP + " << jx << "), o" << iy
+                              << "_" << jx << ");\n";
+                    }
+                }
+                o << ind << "} else {\n";
+                for (int iy = 0; iy < VY; ++iy)
+                    for (int jx = 0; jx < VX; ++jx) {
+                        const std::string gx = "X0 + xt * VX + " + num(jx), gy = "Y0 + by + " + num(iy);
+                        const std::string inb = boxed ? "zin && " + gx + " >= " + BX0 + " && " + gx + " < " +
+                                                            BX1 + " && " + gy + " >= " + BY0 + " && " + gy +
+                                                            " < " + BY1
+                                                      : gx + " < NX && " + gy + " < NY";
+                        o << ind << "  if (" << inb << ") sf_st(" << gbn << " + (" << iy << " * XP + " << jx
+                          << "), o" << iy << "_" << jx << ");\n";
+                    }
+                o << ind << "}\n";
+            };
             o << "          if (zst) {\n";
             o << "            T *const gb = gpl + cg + b * (YT * VY * XP);\n";
-            o << "            if (fast) {\n";
-            for (int iy = 0; iy < VY; ++iy) {
-                if (vec_ok) {
-                    for (int jx = 0; jx < VX; jx += VW) {
-                        o << "              sf_st_v(gb + (" << iy << " * XP + " << jx << "), T2{";
-                        for (int e2 = 0; e2 < VW; ++e2)
-                            o << (e2 ? ", " : "") << "o" << iy << "_" << jx + e2;
-                        o << "});\n";
-                    }
-                } else {
-                    for (int jx = 0; jx < VX; ++jx)
-                        o << "              sf_st(gb + (" << iy << " * XP + " << jx << "), o" << iy
-                          << "_" << jx << ");\n";
+            stores("gb", "            ");
+            for (size_t k = 0; k < L.pushes.size(); ++k) {
+                const Launch::Push &u = L.pushes[k];
+                if (u.stage != (int)m) continue;
+                // the same element of the neighbour's buffer, one slab up/down (layouts are
+                // identical on every rank): its top / bottom ghost planes
+                const std::string off = "(gb - p.arr[" + num(L.arr_slot[G.out]) + "])";
+                if (u.dn > 0) {
+                    o << "            if (gz < " << u.dn << " && p.xp[" << k << "][0]) {  // push down\n";
+                    o << "              T *const pb = p.xp[" << k << "][0] + " << off << " + (long long)NZ * PLANE;\n";
+                    stores("pb", "              ");
+                    o << "            }\n";
+                }
+                if (u.up > 0) {
+                    o << "            if (gz >= NZ - " << u.up << " && p.xp[" << k << "][1]) {  // push up\n";
+                    o << "              T *const pb = p.xp[" << k << "][1] + " << off << " - (long long)NZ * PLANE;\n";
+                    stores("pb", "              ");
+                    o << "            }\n";
                 }
             }
-            o << "            } else {\n";
-            for (int iy = 0; iy < VY; ++iy)
-                for (int jx = 0; jx < VX; ++jx)
-                {
-                    const std::string gx = "X0 + xt * VX + " + num(jx), gy = "Y0 + by + " + num(iy);
-                    const std::string inb = boxed ? "zin && " + gx + " >= " + BX0 + " && " + gx + " < " +
-                                                        BX1 + " && " + gy + " >= " + BY0 + " && " + gy +
-                                                        " < " + BY1
-                                                  : gx + " < NX && " + gy + " < NY";
-                    o << "              if (" << inb << ") sf_st(gb + (" << iy << " * XP + " << jx
-                      << "), o" << iy << "_" << jx << ");\n";
-                }
-            o << "            }\n          }\n";
+            o << "          }\n";
         }
         o << "        }\n";
 
@@ -861,7 +909,17 @@ std::string generate_launch(const stencil_program *p, Launch &L, int index, bool
     } else {
         o << "    sf_bar_sync(1, NT);\n";
     }
-    o << "  }\n}\n";
+    o << "  }\n";
+    if (L.xp) {
+        // completion: the last CTA publishes seq to itself and to both neighbours
+        o << "  __threadfence_system();  // this thread's stores (incl. peer pushes) first\n";
+        o << "  sf_bar_sync(3, NT);\n";
+        if (std::getenv("SF_DEBUG_XP"))
+            o << "  if (tid == 0) printf(\"[" << L.fn << "] own=%p seq=%llu Z0=%d done\\n\", p.xs_own, xs_seq, Z0);\n";
+        o << "  if (tid == 0) sf_xs_signal(p.xs_ctr, gridDim.x * gridDim.y * gridDim.z, p.xs_self, "
+             "p.xs_dn, p.xs_up, xs_seq);\n";
+    }
+    o << "}\n";
     L.source = o.str();
     std::ostringstream tbl;
     tbl << "__constant__ T SFK[" << std::max<size_t>(coefs.size(), 1) << "] = {";

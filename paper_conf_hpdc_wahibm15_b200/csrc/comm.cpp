@@ -12,6 +12,7 @@
 //     ranks publish at host barriers.  It runs the executor's multi-rank schedule
 //     (exchange set, interior/boundary split, events) exactly as NCCL does; only
 //     the wire differs.
+#include <cuda.h>
 #include <cuda_runtime.h>
 #include <nccl.h>
 
@@ -20,6 +21,7 @@
 #include <atomic>
 #include <thread>
 #include <cstring>
+#include <map>
 
 #include "sf_internal.h"
 
@@ -36,6 +38,7 @@ struct LoopHub {
     std::atomic<uint64_t> gen{0};
     std::vector<stencil_program *> prog;
     std::vector<cudaEvent_t> ready, done;
+    std::once_flag events_once;  // created at the first exchange (creation needs no GPU)
 
     // all n virtual ranks meet (spinning: the exchange issues device work between
     // barriers and a sleeping wake-up would starve the GPU); a missing rank (an
@@ -63,20 +66,56 @@ struct LoopHub {
 
 // Per launch, the arrays whose ghost planes must be received before it, with the
 // depth below/above.  An array is exchanged once per "epoch" (the step start or a
-// launch that stores it, up to the next such launch), before the epoch's first
-// launch that reads it beyond the slab, at the largest depth any reader of the
-// epoch needs; an unchanged array is not re-sent to every consumer.  A launch
-// never reads beyond the slab an array it stores (reading R11), so the epoch's
-// value is the one every reader sees.
+// launch that stores it, up to the next such launch), at the largest depth any
+// reader of the epoch needs; an unchanged array is not re-sent to every consumer.
+// An epoch that begins at a store is exchanged before its first launch that reads
+// the array beyond the slab; every step-start epoch (values final before the step:
+// IN arrays, state of the previous step) is exchanged in ONE exchange in front of
+// the step's first launch.  A launch never reads beyond the slab an array it
+// stores (reading R11), so the epoch's value is the one every reader sees.
+//
+// Peer push (option xpush, several ranks): an epoch that begins at a store of a
+// TEMP array is not exchanged at all; the storing launch writes the planes the
+// neighbours' readers need straight into their ghost planes (peer stores over
+// NVLink, or the loopback ranks' buffers), and the kernels order themselves with
+// the neighbours through per-launch progress flags (codegen: xp protocol).  TEMP
+// only: the caller never rebinds scratch arrays, so the neighbours' mapped
+// buffers stay valid across steps.
 void exchange_schedule(const stencil_program *p, Mode &m) {
     const size_t n = m.launches.size();
     const int na = (int)p->arrays.size();
+    const bool push = p->opt.xpush && p->comm && p->comm->nranks > 1;
     m.xsched.assign(n, {});
-    std::vector<int> first(na, -1), below(na, 0), above(na, 0);
+    for (Launch &L : m.launches) {
+        L.pushes.clear();
+        L.xp = push && !L.dead;
+        L.xp_dw = 0;
+    }
+    const bool nowait = p->opt.xpush == 2;  // debugging only: the protocol without waits
+    int first_live = -1;
+    for (size_t i = 0; i < n && first_live < 0; ++i)
+        if (!m.launches[i].dead) first_live = (int)i;
+    std::vector<int> first(na, -1), below(na, 0), above(na, 0), writer(na, -1);
+    std::vector<std::vector<int>> readers(na);
     auto flush = [&](int a) {
-        if (first[a] >= 0) m.xsched[first[a]].push_back({a, below[a], above[a]});
+        if (first[a] >= 0) {
+            if (push && writer[a] >= 0 && p->arrays[a].role == SP_TEMP) {
+                Launch &W = m.launches[writer[a]];
+                for (size_t s = 0; s < W.st.size(); ++s)
+                    if (W.st[s].stored && W.st[s].out == a)
+                        W.pushes.push_back({(int)s, above[a], below[a]});
+                if (!nowait) W.xp_dw = std::max({W.xp_dw, above[a], below[a]});
+                for (int r : (nowait ? std::vector<int>{} : readers[a])) {
+                    Launch &R = m.launches[r];
+                    R.xp_dw = std::max({R.xp_dw, R.z_below, R.z_above});
+                }
+            } else {
+                m.xsched[first[a]].push_back({a, below[a], above[a]});
+            }
+        }
         first[a] = -1;
         below[a] = above[a] = 0;
+        readers[a].clear();
     };
     for (size_t i = 0; i < n; ++i) {
         const Launch &L = m.launches[i];
@@ -84,12 +123,16 @@ void exchange_schedule(const stencil_program *p, Mode &m) {
         for (const Input &I : L.in) {
             const int b = std::max(0, -I.qlo), u = std::max(0, I.ahi);
             if (!b && !u) continue;
-            if (first[I.arr] < 0) first[I.arr] = (int)i;
+            if (first[I.arr] < 0) first[I.arr] = writer[I.arr] >= 0 ? (int)i : first_live;
             below[I.arr] = std::max(below[I.arr], b);
             above[I.arr] = std::max(above[I.arr], u);
+            readers[I.arr].push_back((int)i);
         }
         for (const Stage &G : L.st)
-            if (G.stored) flush(G.out);
+            if (G.stored) {
+                flush(G.out);
+                writer[G.out] = (int)i;
+            }
     }
     for (int a = 0; a < na; ++a) flush(a);
     for (auto &v : m.xsched)
@@ -102,6 +145,15 @@ static void exchange_loopback(stencil_program *p, const std::vector<Mode::Xfer> 
     sp_comm *c = p->comm;
     LoopHub &h = *c->hub;
     const int r = c->rank;
+    std::call_once(h.events_once, [&] {
+        for (int k = 0; k < h.n; ++k)
+            for (auto *v : {&h.ready, &h.done}) {
+                cudaEvent_t e;
+                if (cudaEventCreateWithFlags(&e, cudaEventDisableTiming) != cudaSuccess)
+                    fail(SP_E_CUDA, "cudaEventCreate");
+                v->push_back(e);
+            }
+    });
     h.prog[r] = p;
     if (cudaEventRecord(h.ready[r], s) != cudaSuccess) fail(SP_E_CUDA, "event record");
     h.barrier();  // every rank's slab is final up to its `ready`
@@ -179,6 +231,18 @@ void sf_comm_unique_id_impl(void *out) {
     std::memcpy(out, &id, 128);
 }
 
+namespace sf {
+void *comm_stream(sp_comm *c) {
+    if (!c->comm_stream) {
+        cudaStream_t s;
+        if (cudaStreamCreateWithFlags(&s, cudaStreamNonBlocking) != cudaSuccess)
+            fail(SP_E_CUDA, "cudaStreamCreate (comm stream)");
+        c->comm_stream = s;
+    }
+    return c->comm_stream;
+}
+}  // namespace sf
+
 static cudaStream_t new_stream() {
     cudaStream_t s;
     if (cudaStreamCreateWithFlags(&s, cudaStreamNonBlocking) != cudaSuccess)
@@ -201,25 +265,17 @@ sp_comm *sf_comm_create_impl(const void *idp, int32_t nranks, int32_t rank) {
     return c.release();
 }
 
+// no CUDA call here: streams and events are created at the first exchange, so a
+// loopback program can be analysed and JIT-compiled on a host without a GPU
 void sf_comm_create_loopback_impl(int32_t nranks, sp_comm **out) {
-    sf::ensure_cuda();
     auto hub = std::make_shared<sf::LoopHub>();
     hub->n = nranks;
     hub->prog.assign(nranks, nullptr);
-    for (int r = 0; r < nranks; ++r)
-        for (auto *v : {&hub->ready, &hub->done}) {
-            cudaEvent_t e;
-            if (cudaEventCreateWithFlags(&e, cudaEventDisableTiming) != cudaSuccess)
-                sf::fail(SP_E_CUDA, "cudaEventCreate");
-            v->push_back(e);
-        }
     std::vector<std::unique_ptr<sp_comm>> cs;
     for (int r = 0; r < nranks; ++r) {
         std::unique_ptr<sp_comm> c(new sp_comm());
         c->nranks = nranks;
         c->rank = r;
-        cudaGetDevice(&c->device);
-        c->comm_stream = new_stream();
         c->hub = hub;
         cs.push_back(std::move(c));
     }
@@ -230,4 +286,36 @@ void sf_comm_destroy_impl(sp_comm *c) {
     if (c->nccl) ncclCommDestroy((ncclComm_t)c->nccl);
     if (c->comm_stream) cudaStreamDestroy((cudaStream_t)c->comm_stream);
     delete c;
+}
+
+// CUDA IPC of a device pointer inside a cudaMalloc allocation (e.g. a torch
+// tensor of the caching allocator): the handle names the whole allocation, the
+// offset the pointer inside it.  A process opens each allocation once.
+void sf_ipc_export_impl(const void *ptr, void *handle64, int64_t *offset) {
+    static_assert(sizeof(cudaIpcMemHandle_t) == 64, "cudaIpcMemHandle_t size");
+    CUdeviceptr base = 0;
+    size_t size = 0;
+    if (!sf::driver_mem_range(&base, &size, (CUdeviceptr)ptr))
+        sf::fail(SP_E_CUDA, "cuMemGetAddressRange");
+    cudaIpcMemHandle_t h;
+    if (cudaIpcGetMemHandle(&h, (void *)base) != cudaSuccess) sf::fail(SP_E_CUDA, "cudaIpcGetMemHandle");
+    std::memcpy(handle64, &h, 64);
+    *offset = (int64_t)((CUdeviceptr)ptr - base);
+}
+
+void *sf_ipc_open_impl(const void *handle64, int64_t offset) {
+    static std::mutex mu;
+    static std::map<std::string, void *> opened;
+    std::lock_guard<std::mutex> lk(mu);
+    std::string key((const char *)handle64, 64);
+    auto it = opened.find(key);
+    if (it == opened.end()) {
+        cudaIpcMemHandle_t h;
+        std::memcpy(&h, handle64, 64);
+        void *base = nullptr;
+        if (cudaIpcOpenMemHandle(&base, h, cudaIpcMemLazyEnablePeerAccess) != cudaSuccess)
+            sf::fail(SP_E_CUDA, "cudaIpcOpenMemHandle");
+        it = opened.emplace(key, base).first;
+    }
+    return (char *)it->second + offset;
 }

@@ -148,3 +148,50 @@ __device__ __forceinline__ float sf_ld(const float *p) {
     asm volatile("ld.global.nc.f32 %0, [%1];" : "=f"(v) : "l"(p));
     return v;
 }
+
+// ---- peer-push halo protocol (several ranks, option xpush) --------------------
+// Signal block of a rank (64 B, device memory of that rank, mapped by its
+// neighbours): u64 [0] progress published by the lower neighbour, [1] by the
+// upper neighbour, [2] this rank's own progress; u32 at byte 24: CTAs done.
+__device__ __forceinline__ sf_u64 sf_ld_volatile_u64(const sf_u64 *p) {
+    sf_u64 v;
+    asm volatile("ld.volatile.global.u64 %0, [%1];" : "=l"(v) : "l"(p) : "memory");
+    return v;
+}
+__device__ __forceinline__ sf_u64 sf_ld_acquire_sys(const sf_u64 *p) {
+    sf_u64 v;
+    asm volatile("ld.acquire.sys.global.u64 %0, [%1];" : "=l"(v) : "l"(p) : "memory");
+    return v;
+}
+__device__ __forceinline__ void sf_st_release_sys(sf_u64 *p, sf_u64 v) {
+    asm volatile("st.release.sys.global.u64 [%0], %1;" ::"l"(p), "l"(v) : "memory");
+}
+__device__ __forceinline__ sf_u64 sf_globaltimer() {
+    sf_u64 t;
+    asm volatile("mov.u64 %0, %globaltimer;" : "=l"(t));
+    return t;
+}
+// wait until the existing neighbours have published progress >= want; a peer that
+// never arrives (a rank that stopped) traps after 20 s instead of hanging the GPU
+__device__ __forceinline__ void sf_xs_wait(const sf_u64 *own, bool has_dn, bool has_up, sf_u64 want) {
+    const sf_u64 t0 = sf_globaltimer();
+    while ((has_dn && sf_ld_acquire_sys(own + 0) < want) || (has_up && sf_ld_acquire_sys(own + 1) < want)) {
+        asm volatile("nanosleep.u32 200;");
+        if (sf_globaltimer() - t0 > 20000000000ull) asm volatile("trap;");
+    }
+    // the pushed planes were written through the generic proxy; TMA reads them
+    asm volatile("fence.proxy.async.global;" ::: "memory");
+}
+// CTA completion; the last CTA of the grid publishes seq (own progress and both
+// neighbours' "from" slots) after a system-scope fence
+__device__ __forceinline__ void sf_xs_signal(sf_u32 *ctr, sf_u32 total, sf_u64 *self, sf_u64 *dn,
+                                             sf_u64 *up, sf_u64 seq) {
+    sf_u32 old;
+    asm volatile("atom.acq_rel.gpu.global.add.u32 %0, [%1], 1;" : "=r"(old) : "l"(ctr) : "memory");
+    if (old != total - 1) return;
+    asm volatile("st.relaxed.gpu.global.u32 [%0], 0;" ::"l"(ctr) : "memory");
+    asm volatile("fence.sc.sys;" ::: "memory");
+    asm volatile("st.volatile.global.u64 [%0], %1;" ::"l"(self), "l"(seq) : "memory");
+    if (dn) sf_st_release_sys(dn + 1, seq);  // I am the lower neighbour's upper neighbour
+    if (up) sf_st_release_sys(up + 0, seq);
+}

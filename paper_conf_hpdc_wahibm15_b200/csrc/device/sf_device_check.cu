@@ -31,3 +31,15 @@ extern "C" __global__ void __launch_bounds__(128)
     }
     sf_st(out + blockIdx.x * 128 + threadIdx.x, acc);
 }
+
+// the peer-push protocol primitives (wait on the neighbours, last-CTA signal)
+extern "C" __global__ void __launch_bounds__(32)
+    sf_device_check_xs(sf_u64 *sig, sf_u64 *dn, sf_u64 *up, double *peer, double v) {
+    const sf_u64 seq = sf_ld_volatile_u64(sig + 2) + 1;
+    if (threadIdx.x == 0) sf_xs_wait(sig, dn != nullptr, up != nullptr, seq - 1);
+    __syncthreads();
+    sf_st(peer + threadIdx.x, v);
+    __threadfence_system();
+    __syncthreads();
+    if (threadIdx.x == 0) sf_xs_signal((sf_u32 *)(sig + 3), gridDim.x, sig + 2, dn, up, seq);
+}

@@ -42,7 +42,8 @@ struct Drv {
                                      CUtensorMapFloatOOBfill) = nullptr;
     CUresult (*GetErrorString)(CUresult, const char **) = nullptr;
     CUresult (*LaunchKernelEx)(const CUlaunchConfig *, CUfunction, void **, void **) = nullptr;
-    bool ok = false;
+    CUresult (*MemGetAddressRange)(CUdeviceptr *, size_t *, CUdeviceptr) = nullptr;
+    std::atomic<bool> ok{false};
 };
 static Drv g_drv;
 static std::mutex g_drv_mu;
@@ -71,14 +72,17 @@ static void entry(const char *name, F &fp) {
 }
 
 void ensure_cuda() {
+    // fast path: no runtime call (cudaFree(0) may synchronize the device, which a
+    // rank whose kernels wait on a neighbour's progress must never do mid-step)
+    if (g_drv.ok) return;
     std::lock_guard<std::mutex> lk(g_drv_mu);
+    if (g_drv.ok) return;
     int n = 0;
     cudaError_t e = cudaGetDeviceCount(&n);
     if (e != cudaSuccess || n == 0)
         fail(SP_E_CUDA, std::string("no CUDA device available (") + cudaGetErrorString(e) +
                             "); this library has no CPU fallback");
     cuda_check(cudaFree(nullptr), "cudaFree(0) (context init)");
-    if (g_drv.ok) return;
     entry("cuModuleLoadData", g_drv.ModuleLoadData);
     entry("cuModuleUnload", g_drv.ModuleUnload);
     entry("cuModuleGetFunction", g_drv.ModuleGetFunction);
@@ -88,7 +92,13 @@ void ensure_cuda() {
     entry("cuTensorMapEncodeTiled", g_drv.TensorMapEncodeTiled);
     entry("cuGetErrorString", g_drv.GetErrorString);
     entry("cuLaunchKernelEx", g_drv.LaunchKernelEx);
+    entry("cuMemGetAddressRange", g_drv.MemGetAddressRange);
     g_drv.ok = true;
+}
+
+bool driver_mem_range(CUdeviceptr *base, size_t *size, CUdeviceptr p) {
+    ensure_cuda();
+    return g_drv.MemGetAddressRange(base, size, p) == CUDA_SUCCESS;
 }
 
 // ------------------------------------------------------------------ NVRTC
@@ -218,6 +228,18 @@ void load_mode(stencil_program *p, Mode &m) {
     m.loaded = true;
 }
 
+void *signal_block(stencil_program *p) {
+    if (!p->sig) {
+        ensure_cuda();
+        void *s = nullptr;
+        if (cudaMalloc(&s, 64) != cudaSuccess || cudaMemset(s, 0, 64) != cudaSuccess ||
+            cudaDeviceSynchronize() != cudaSuccess)
+            fail(SP_E_CUDA, "signal block allocation");
+        p->sig = s;
+    }
+    return p->sig;
+}
+
 static void build_params(stencil_program *p, Mode &m) {
     if (m.maps_version == p->bind_version) return;
     const int e = p->elem;
@@ -250,6 +272,33 @@ static void build_params(stencil_program *p, Mode &m) {
             void *ptr = p->ptrs[L.slot_arr[s]];
             if (!ptr) fail(SP_E_STATE, "array '" + p->arrays[L.slot_arr[s]].name + "' is not bound");
             std::memcpy(buf + L.ptr_off + 8 * s, &ptr, 8);
+        }
+        if (L.xp) {
+            // peer-push section: own signal block, neighbours' blocks and buffers
+            // (a missing neighbour — rank 0 below, the last rank above — stays null)
+            const int r = p->comm->rank, nr = p->comm->nranks;
+            const bool has[2] = {r > 0, r + 1 < nr};
+            // (allocated by sp_signal_buffer when the peers are wired: allocating here,
+            // mid-step, could synchronise the device under a waiting neighbour)
+            if (!p->sig) fail(SP_E_STATE, "peer push: no signal block (sp_signal_buffer)");
+            char *sig = (char *)p->sig;
+            void *v[5] = {sig + 16, sig, has[0] ? p->peer_sig[0] : nullptr,
+                          has[1] ? p->peer_sig[1] : nullptr, sig + 24};
+            for (int s = 0; s < 2; ++s)
+                if (has[s] && !p->peer_sig[s])
+                    fail(SP_E_STATE, "peer push: the neighbours' signal blocks are not bound "
+                                     "(sp_bind_peer_signal)");
+            std::memcpy(buf + L.xp_off, v, 40);
+            for (size_t k = 0; k < L.pushes.size(); ++k) {
+                const int a = L.st[L.pushes[k].stage].out;
+                for (int s = 0; s < 2; ++s) {
+                    void *q = has[s] ? p->peer[a][s] : nullptr;
+                    if (has[s] && !q)
+                        fail(SP_E_STATE, "peer push: neighbour buffer of '" + p->arrays[a].name +
+                                             "' is not bound (sp_bind_peer)");
+                    std::memcpy(buf + L.xp_off + 40 + 16 * k + 8 * s, &q, 8);
+                }
+            }
         }
     }
     m.maps_version = p->bind_version;

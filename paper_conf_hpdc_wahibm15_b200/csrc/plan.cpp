@@ -566,9 +566,9 @@ void analyze_mode(stencil_program *p, bool fused, const std::vector<std::vector<
         }
         m.launches.push_back(std::move(L));
     }
+    exchange_schedule(p, m);  // also decides the peer pushes codegen emits
     for (size_t i = 0; i < m.launches.size(); ++i)
         if (!m.launches[i].dead) generate_launch(p, m.launches[i], (int)i, fused);
-    exchange_schedule(p, m);
     m.analyzed = true;
     out = std::move(m);
 }

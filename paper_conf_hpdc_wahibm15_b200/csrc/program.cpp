@@ -207,6 +207,7 @@ stencil_program *sf_program_create_impl(const sp_grid *grid, int32_t n_arrays,
     p->zint_lo = -g.z_offset;
     p->zint_hi = g.nz_global - g.z_offset;
     p->ptrs.assign(n_arrays, nullptr);
+    p->peer.assign(n_arrays, {nullptr, nullptr});
     build_edges(p.get());
     return p.release();
 }

@@ -7,6 +7,7 @@
 #pragma once
 
 #include <cstdint>
+#include <array>
 #include <map>
 #include <memory>
 #include <mutex>
@@ -43,6 +44,7 @@ struct Options {
     int factor = 1;     // perf build: terms sharing one b operand are summed, then multiplied once
     int zwave = 0;          // z-wave schedule: planes per wave (0 = one launch per group per step)
     int zwave_streams = 2;  // waves in flight (streams) of the z-wave schedule
+    int xpush = 0;  // several ranks: stores push in-step halo planes into the neighbours' ghosts
 };
 
 // ---------------------------------------------------------------- analysis
@@ -118,6 +120,14 @@ struct Launch {
     void *func = nullptr;    // CUfunction
     void *module = nullptr;  // CUmodule
     size_t param_size = 0, ptr_off = 0, int_off = 0;
+    // peer-push halo exchange (option xpush, several ranks): stage `stage` also stores
+    // its bottom `dn` planes into the lower neighbour's top ghost and its top `up`
+    // planes into the upper neighbour's bottom ghost
+    struct Push { int stage, dn, up; };
+    std::vector<Push> pushes;
+    bool xp = false;         // kernel carries the peer-push signal protocol
+    int xp_dw = 0;           // chunks within xp_dw planes of a slab end wait for the neighbours
+    size_t xp_off = 0;       // param offset of the peer-push section
     bool dead = false;       // nothing to compute (all stages dead)
     bool pdl = false;        // launched with programmatic stream serialization
 };
@@ -169,6 +179,12 @@ struct stencil_program_s {
     bool no_pdl = false;         // multi-rank schedule: plain stream order between launches
     std::vector<void *> wave_streams, wave_events;  // z-wave schedule: streams, events
     std::map<int, sp_tile_config> tune_fused, tune_unfused;  // sp_plan_tune overrides
+    // peer-push exchange: neighbours' buffers of each array (0 = below, 1 = above),
+    // this program's signal block (u64 from_dn, from_up, self; u32 cta counter) and
+    // the neighbours' signal blocks, all mapped in this process
+    std::vector<std::array<void *, 2>> peer;
+    void *sig = nullptr;
+    void *peer_sig[2] = {nullptr, nullptr};
 };
 
 namespace sf {
@@ -201,6 +217,8 @@ void load_mode(stencil_program *p, Mode &m);
 void launch(stencil_program *p, Mode &m, int i, void *stream, int z0 = 0, int z1 = -1, int z2 = 0,
             int z3 = 0);
 void ensure_cuda();
+void *signal_block(stencil_program *p);  // allocated (zeroed) on first use
+bool driver_mem_range(unsigned long long *base, size_t *size, unsigned long long p);  // cuMemGetAddressRange
 void unload_mode(Mode &m);
 
 // comm.cpp
@@ -208,4 +226,5 @@ void unload_mode(Mode &m);
 // ghost of each array (the neighbours send the matching interior planes)
 void exchange(stencil_program *p, const std::vector<Mode::Xfer> &x, void *stream);
 void exchange_schedule(const stencil_program *p, Mode &m);
+void *comm_stream(sp_comm *c);  // the communicator's exchange stream (created on first use)
 }  // namespace sf

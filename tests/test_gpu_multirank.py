@@ -111,7 +111,7 @@ def test_virtual_ranks_bitexact(cuda_device, cfg, ranks, fmad):
 @pytest.mark.parametrize("cfg,ranks,mode", [("C2", 2, "fused"), ("C5", 3, "fused"), ("C3", 2, "fused"),
                                             ("C4", 2, "fused"), ("C4", 3, "unfused"),
                                             ("chain3", 3, "fused"), ("C2box", 2, "fused"),
-                                            ("C2", 3, "unfused")])
+                                            ("C2", 3, "unfused"), ("C4", 4, "fused")])
 def test_loopback_ranks_run_bitexact(cuda_device, cfg, ranks, mode):
     """The executor's own multi-rank path (run_fused / run_unfused with a communicator:
     exchange schedule, interior planes overlapped with the exchange on the comm stream,
@@ -146,7 +146,7 @@ def test_loopback_ranks_run_bitexact(cuda_device, cfg, ranks, mode):
         s.set_plan(plan)
         s.allocate(dev)
         fill(s, loc, dev, r * nzl, zhalo, nz_global=nzl * ranks)
-        s.compile(mode)
+        s.load(mode)  # no module load mid-step (see sp_load)
         slabs.append(s)
     torch.cuda.synchronize()
     errs = []
@@ -172,3 +172,80 @@ def test_loopback_ranks_run_bitexact(cuda_device, cfg, ranks, mode):
         want = single.interior_view(single.tensors[n])
         got = torch.cat([s.interior_view(s.tensors[n]) for s in slabs], dim=0)
         assert torch.equal(got, want), f"{cfg} {n}: loopback multi-rank result differs from single domain"
+
+
+MK = {"C2": lambda nz: P.c2(nx=40, ny=24, nz=nz), "C5": lambda nz: P.c5(nx=32, ny=16, nz=nz),
+      "C3": lambda nz: P.c3(nx=48, ny=20, nz=nz), "C4": c4_small,
+      "chain3": lambda nz: P.resize(P.chain3(), 20, 12, nz), "C2box": c2_boxed}
+
+
+@pytest.mark.parametrize("cfg,ranks,mode", [("C3", 2, "fused"), ("C3", 3, "unfused"), ("C4", 2, "fused"),
+                                            ("C4", 3, "fused"), ("C4", 2, "unfused"),
+                                            ("chain3", 3, "unfused"), ("C2", 2, "unfused"),
+                                            ("C2box", 3, "unfused")])
+def test_peer_push_lockstep_bitexact(cuda_device, cfg, ranks, mode):
+    """Peer-push halo exchange (option xpush, NEXT #2) on virtual ranks: every TEMP
+    epoch travels as peer stores from the producing kernel into the neighbours' ghost
+    planes, and every kernel runs the progress protocol (edge chunks wait until both
+    neighbours completed the previous launch; the last CTA publishes completion).
+    One GPU cannot run ranks whose kernels wait on each other concurrently without
+    risking a shared hardware queue (a waiting kernel queued ahead of the work it
+    waits for), so the ranks' launches are issued in lockstep on one stream — a
+    valid schedule of the protocol, in which every wait is already satisfied.  The
+    step-start epochs (IN arrays) are copied as sp_plan_exchange names them.  Two
+    steps; bit-exact with the single domain (P9)."""
+    import torch
+    from paper_conf_hpdc_wahibm15_b200 import Comm, Program
+    nzl = 12
+    mk = MK[cfg]
+    glob = mk(nzl * ranks)
+    plan = glob["plans"]["fused"]
+    dev = cuda_device
+    single = Program(glob)
+    single.set_plan(plan)
+    single.allocate(dev)
+    fill(single, glob, dev, 0, glob["grid"]["ghost"][2])
+    single.run(mode)
+    loc = mk(nzl)
+    probe = Program(loc, nz_global=nzl * ranks)
+    probe.set_plan(plan)
+    zhalo = max([max(r["z_below"], r["z_above"]) for m in ("fused", "unfused")
+                 for r in probe.reports(m)] + [loc["grid"]["ghost"][2]])
+    comms = Comm.loopback(ranks)
+    slabs = []
+    for r in range(ranks):
+        s = Program(loc, comm=comms[r], nz_global=nzl * ranks, z_offset=r * nzl, zhalo=zhalo,
+                    options={"xpush": 1})
+        s.set_plan(plan)
+        s.allocate(dev)
+        fill(s, loc, dev, r * nzl, zhalo, nz_global=nzl * ranks)
+        s.load(mode)
+        slabs.append(s)
+    Program.connect_peers_local(slabs)
+    n = slabs[0].n_launches(mode)
+    nopush = Program(loc, comm=comms[0], nz_global=nzl * ranks, zhalo=zhalo)
+    nopush.set_plan(plan)
+    xfers = [slabs[0].exchange_plan(mode, i) for i in range(n)]
+    # TEMP epochs left the communicator's schedule (they are pushed)
+    temps = {a["name"] for a in loc["arrays"] if a["role"] == "temp"}
+    assert not any(a in temps for x in xfers for a, _, _ in x)
+    if cfg in ("C4", "C3", "chain3"):
+        assert sum(map(len, xfers)) < sum(len(nopush.exchange_plan(mode, i)) for i in range(n))
+    torch.cuda.synchronize()
+    for step in range(2):
+        for i in range(n):
+            for a, below, above in xfers[i]:
+                for r in range(ranks - 1):
+                    lo, hi = slabs[r], slabs[r + 1]
+                    if below:
+                        plane(hi, hi.tensors[a], -below, below).copy_(plane(lo, lo.tensors[a], nzl - below, below))
+                    if above:
+                        plane(lo, lo.tensors[a], nzl, above).copy_(plane(hi, hi.tensors[a], 0, above))
+            for s in slabs:
+                s.run_launch(mode, i)
+    torch.cuda.synchronize()
+    outs = [a["name"] for a in glob["arrays"] if a["role"] in ("out", "inout")]
+    for nm in outs:
+        want = single.interior_view(single.tensors[nm])
+        got = torch.cat([s.interior_view(s.tensors[nm]) for s in slabs], dim=0)
+        assert torch.equal(got, want), f"{cfg} {nm}: peer-push multi-rank result differs from single domain"

@@ -272,8 +272,10 @@ def test_exchange_schedule_matches_reach():
     prog = P.c3(n=32)
     p = Program(prog, nz_global=64, z_offset=0, zhalo=5)
     p.set_plan(prog["plans"]["fission_fused"])
-    assert p.exchange_plan("fused", 0) == [("A", 5, 5)]   # 7pt, 7pt, 13pt, 7pt chain: 1+1+2+1
-    assert p.exchange_plan("fused", 1) == [("B", 5, 5)]   # O1 is read point-wise: no exchange
+    # IN arrays (step-start epochs) all travel in one exchange in front of the first launch;
+    # 7pt, 7pt, 13pt, 7pt chain: reach 1+1+2+1
+    assert p.exchange_plan("fused", 0) == [("A", 5, 5), ("B", 5, 5)]
+    assert p.exchange_plan("fused", 1) == []
     # unfused: each array once per epoch (after its writer), before its first halo reader
     want = {0: [("A", 1, 1), ("B", 1, 1)], 1: [("P", 1, 1)], 2: [("P1", 2, 2)], 3: [("P2", 1, 1)],
             4: [("Q", 1, 1)], 5: [("Q1", 2, 2)], 6: [("Q2", 1, 1)], 7: []}

@@ -52,7 +52,7 @@ def time_ranks(prog, plan, tuned, P, steps, warmup, dev, mode):
                     p.tune("fused", i, c)
         p.allocate(dev, fill=0.0)
         bench.fill_inputs(p, loc, dev, r * nz, zhalo)
-        p.compile(mode)
+        p.load(mode)
         progs.append(p)
     torch.cuda.synchronize()
     out = [0.0] * P

@@ -175,11 +175,15 @@ def run_ours(args):
     zhalo = reach if world > 1 else prog["grid"]["ghost"][2]
     del probe
     comm = Comm(rank, world) if world > 1 else None
-    p = Program(prog, comm=comm, nz_global=nz * world, z_offset=rank * nz, zhalo=zhalo)
+    xpush = bool(args.xpush and world > 1)
+    p = Program(prog, comm=comm, nz_global=nz * world, z_offset=rank * nz, zhalo=zhalo,
+                options={"xpush": 1} if xpush else None)
     p.set_plan(plan)
     apply_tuning(p, prog, args.plan)
     p.allocate(dev, fill=0.0)
     fill_inputs(p, prog, dev, rank * nz, zhalo)
+    if xpush:
+        p.connect_peers(rank, world)
     stream = torch.cuda.current_stream(dev)
     n_pts = prog["grid"]["nx"] * prog["grid"]["ny"] * nz  # per GPU
     n_kernels = len(prog["kernels"])
@@ -336,6 +340,8 @@ def run_ours(args):
                        "kernels": n_kernels, "arrays": len(prog["arrays"]),
                        "plan": args.plan, "fused_groups": len(live_f),
                        "parallelism": f"z-slab x{world}",
+                       "halo_exchange": ("peer-push (TEMP) + NCCL (step-start)" if xpush else
+                                         "NCCL send/recv") if world > 1 else "none",
                        "l2": "no flush: per-GPU working set > 126 MB L2"},
             "hbm_gbs_alg": alg_step / (step_ms * 1e-3) / 1e9,
             "roofline_step": {"achieved": alg_step / (step_ms * 1e-3) / 1e9, "peak": peak,
@@ -434,6 +440,9 @@ def main():
     ap.add_argument("--impl", default="ours", choices=["ours", "reference"])
     ap.add_argument("--plan", default="fused", help="named plan of the workload (e.g. C3 fission_fused)")
     ap.add_argument("--no-cpu", action="store_true", help="skip the cpu_baseline leg")
+    ap.add_argument("--xpush", action="store_true",
+                    help="N > 1: peer-push halo exchange of TEMP epochs (CUDA IPC over NVLink, "
+                         "in-kernel progress protocol) instead of NCCL send/recv for them")
     args = ap.parse_args()
     if args.warmup < 3:
         args.warmup = 3

@@ -249,3 +249,123 @@ def test_peer_push_lockstep_bitexact(cuda_device, cfg, ranks, mode):
         want = single.interior_view(single.tensors[nm])
         got = torch.cat([s.interior_view(s.tensors[nm]) for s in slabs], dim=0)
         assert torch.equal(got, want), f"{cfg} {nm}: peer-push multi-rank result differs from single domain"
+
+
+def _ipc_worker(rank, world, port, cfg, q, concurrent=False):
+    """One process per virtual rank on the same GPU: peer buffers and signal blocks
+    wired through CUDA IPC (Program.connect_peers over gloo).  Lockstep: launch i of
+    rank r runs after launch i of ranks < r and launch i-1 of all.  Concurrent: after
+    the step-start exchange each process enqueues its whole step at once and the
+    kernels order themselves through the in-kernel progress protocol (the two
+    contexts time-slice the GPU, so a waiting kernel is preempted, not a deadlock)."""
+    import sys
+    root = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+    sys.path.insert(0, root)
+    sys.path.insert(0, os.path.join(root, "tests"))
+    import torch
+    import torch.distributed as dist
+    os.environ["MASTER_ADDR"] = "127.0.0.1"
+    os.environ["MASTER_PORT"] = str(port)
+    dist.init_process_group("gloo", rank=rank, world_size=world)
+    try:
+        from paper_conf_hpdc_wahibm15_b200 import Comm, Program
+        from test_gpu_multirank import MK, fill, plane
+        dev = torch.device("cuda:0")
+        torch.cuda.set_device(dev)
+        nzl, mode = 12, "fused"
+        loc = MK[cfg](nzl)
+        plan = loc["plans"]["fused"]
+        probe = Program(loc, nz_global=nzl * world)
+        probe.set_plan(plan)
+        zhalo = max([max(r["z_below"], r["z_above"]) for m in ("fused", "unfused")
+                     for r in probe.reports(m)] + [loc["grid"]["ghost"][2]])
+        comm = Comm.loopback(world)[rank]  # only its rank count is used (no run_fused here)
+        s = Program(loc, comm=comm, nz_global=nzl * world, z_offset=rank * nzl, zhalo=zhalo,
+                    options={"xpush": 1})
+        s.set_plan(plan)
+        s.allocate(dev)
+        fill(s, loc, dev, rank * nzl, zhalo, nz_global=nzl * world)
+        s.load(mode)
+        s.connect_peers(rank, world)
+        torch.cuda.synchronize()
+        n = s.n_launches(mode)
+        for step in range(2):
+            for i in range(n):
+                for a, below, above in s.exchange_plan(mode, i):  # step-start epochs over gloo
+                    t = s.tensors[a]
+                    if rank + 1 < world:
+                        if below:
+                            dist.send(plane(s, t, nzl - below, below).cpu().contiguous(), dst=rank + 1)
+                        if above:
+                            buf = torch.empty_like(plane(s, t, 0, above), device="cpu")
+                            dist.recv(buf, src=rank + 1)
+                            plane(s, t, nzl, above).copy_(buf)
+                    if rank > 0:
+                        if below:
+                            buf = torch.empty_like(plane(s, t, 0, below), device="cpu")
+                            dist.recv(buf, src=rank - 1)
+                            plane(s, t, -below, below).copy_(buf)
+                        if above:
+                            dist.send(plane(s, t, 0, above).cpu().contiguous(), dst=rank - 1)
+                if concurrent:
+                    if i == 0:
+                        torch.cuda.synchronize()
+                        dist.barrier()
+                    s.run_launch(mode, i)
+                    continue
+                torch.cuda.synchronize()
+                dist.barrier()
+                for r in range(world):
+                    if r == rank:
+                        s.run_launch(mode, i)
+                        torch.cuda.synchronize()
+                    dist.barrier()
+            assert all(not x for i in range(1, n) for x in s.exchange_plan(mode, i)) or not concurrent
+            torch.cuda.synchronize()
+            dist.barrier()
+        outs = [a["name"] for a in loc["arrays"] if a["role"] in ("out", "inout")]
+        mine = {nm: s.interior_view(s.tensors[nm]).cpu() for nm in outs}
+        got = [None] * world if rank == 0 else None
+        dist.gather_object(mine, got, dst=0)
+        if rank == 0:
+            glob = MK[cfg](nzl * world)
+            single = Program(glob)
+            single.set_plan(plan)
+            single.allocate(dev)
+            fill(single, glob, dev, 0, glob["grid"]["ghost"][2])
+            single.run(mode)
+            torch.cuda.synchronize()
+            for nm in outs:
+                want = single.interior_view(single.tensors[nm]).cpu()
+                have = torch.cat([g[nm] for g in got], dim=0)
+                assert torch.equal(have, want), f"{cfg} {nm}: IPC peer-push result differs"
+        q.put((rank, "ok"))
+    except Exception as e:  # surfaced in the parent
+        import traceback
+        q.put((rank, traceback.format_exc()))
+    finally:
+        dist.destroy_process_group()
+
+
+@pytest.mark.parametrize("cfg,concurrent", [("C4", False), ("C3", False), ("C4", True), ("C3", True)])
+def test_peer_push_ipc_processes(cuda_device, cfg, concurrent):
+    """Peer push across PROCESSES (the real deployment shape: one process per rank):
+    each rank maps its neighbours' TEMP buffers and signal blocks with CUDA IPC
+    (sp_ipc_export / sp_ipc_open via Program.connect_peers).  Both processes share
+    one GPU here; their launches run in lockstep.  Bit-exact with the single domain."""
+    import multiprocessing as mp
+    import socket
+    sk = socket.socket()
+    sk.bind(("127.0.0.1", 0))
+    port = sk.getsockname()[1]
+    sk.close()
+    ctx = mp.get_context("spawn")
+    q = ctx.Queue()
+    world = 2
+    ps = [ctx.Process(target=_ipc_worker, args=(r, world, port, cfg, q, concurrent)) for r in range(world)]
+    for p in ps:
+        p.start()
+    res = dict(q.get(timeout=300) for _ in range(world))
+    for p in ps:
+        p.join(timeout=60)
+    assert all(v == "ok" for v in res.values()), res

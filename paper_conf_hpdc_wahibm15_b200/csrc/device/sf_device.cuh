@@ -125,7 +125,8 @@ __device__ __forceinline__ void sf_st_v(float *p, float4 v) {
 }
 
 // ghost value of a point outside the global interior: predicated non-coherent
-// load (ghost cells are never written), 0 when the point is outside the allocation
+// load (no kernel writes ghost cells of the arrays it reads while it runs), 0 when
+// the point is outside the allocation
 __device__ __forceinline__ double sf_ldg_pred(const double *p, bool pred) {
     double v = 0.0;
     asm("{\n\t.reg .pred P1;\n\tsetp.ne.b32 P1, %2, 0;\n\t@P1 ld.global.nc.f64 %0, [%1];\n}"

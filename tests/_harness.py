@@ -76,3 +76,25 @@ def assert_close(prog, got, ref, exact=False):
         else:
             e = rel_err(got[name], ref[name])
             assert e <= tolerance(prog["dtype"]), f"{name}: rel err {e}"
+
+
+def window_field(seed, aid, origin, n, h, dtype):
+    """Generated values (synth/fields.py recipe) of one array on the window whose interior
+    starts at global `origin`, with ghost width h: the same numbers the GPU slab holds."""
+    from synth.fields import bits_to_unit, pack, seed_mix, splitmix64
+    i = np.arange(origin[0] - h[0], origin[0] + n[0] + h[0], dtype=np.int64)
+    j = np.arange(origin[1] - h[1], origin[1] + n[1] + h[1], dtype=np.int64)
+    k = np.arange(origin[2] - h[2], origin[2] + n[2] + h[2], dtype=np.int64)
+    key = pack(i[None, None, :], j[None, :, None], k[:, None, None])
+    return np.ascontiguousarray(bits_to_unit(splitmix64(key ^ seed_mix(seed, aid)), dtype))
+
+
+def accumulated_reach(prog):
+    """Per axis, the sum over kernels of each kernel's largest tap offset: a window of the
+    grid evaluated alone is exact this far inside its edges (conservative)."""
+    m = [0, 0, 0]
+    for k in prog["kernels"]:
+        for d in range(3):
+            m[d] += max(abs(t[x][1 + d]) for s in k["stmts"] for t in s["terms"]
+                        for x in ("a", "b") if x in t)
+    return m

@@ -197,3 +197,49 @@ def test_zwave_full_size_c4(cuda_device):
         outs[zw] = gpu_run(prog, "fused", 9, program=p, repeat=2)
     for n in outs[0]:
         assert outs[0][n].tobytes() == outs[32][n].tobytes(), n
+
+
+@pytest.mark.parametrize("workload,plan,w", [("C5", "fused", 24), ("C3", "measured", 32),
+                                             ("C3", "fission_fused", 32)])
+def test_full_size_sampled_bench_configuration(cuda_device, workload, plan, w):
+    """BASELINE configs[2] (C3, 512^3 fp32) and configs[4]'s per-GPU grid (C5, 1024x1024x128
+    fp64) at full size, in the launch configuration bench.py times (plan + tuned tiles,
+    perf build), checked on sampled windows the oracle evaluates one by one: corner,
+    centre and far-corner windows of w^3 points; inside the window the oracle runs the
+    whole program, and its result is exact wherever the window's margin covers the
+    program's accumulated reach m (compared there; sides on the global boundary need no
+    margin: their ghosts are the true ghosts, reading R1)."""
+    import sys
+    import torch
+    sys.path.insert(0, os.path.dirname(os.path.dirname(os.path.abspath(__file__))))
+    import bench
+    from _harness import accumulated_reach, gpu_program, rel_err, tolerance, window_field
+    from oracle import OracleProgram
+    prog = bench.load_workload(workload)
+    g = prog["grid"]
+    N = (g["nx"], g["ny"], g["nz"])
+    h = tuple(g["ghost"])
+    m = accumulated_reach(prog)
+    p = gpu_program(prog, plan=bench.plan_of(prog, plan))
+    bench.apply_tuning(p, prog, plan)
+    dev = torch.device("cuda:0")
+    p.allocate(dev, fill=0.0)
+    bench.fill_inputs(p, prog, dev, 0, h[2])
+    p.run_fused()
+    torch.cuda.synchronize()
+    outs = [a["name"] for a in prog["arrays"] if a["role"] in ("out", "inout")]
+    orc = OracleProgram(prog)
+    for origin in [(0, 0, 0), tuple((N[d] - w) // 2 for d in range(3)), tuple(N[d] - w for d in range(3))]:
+        win = {a["name"]: window_field(4, aid, origin, (w, w, w), h, prog["dtype"])
+               for aid, a in enumerate(prog["arrays"])}
+        orc.run(win, n=(w, w, w), origin=origin)
+        lo = [origin[d] + (m[d] if origin[d] > 0 else 0) for d in range(3)]
+        hi = [origin[d] + w - (m[d] if origin[d] + w < N[d] else 0) for d in range(3)]
+        assert all(hi[d] > lo[d] for d in range(3)), (lo, hi)
+        for nm in outs:
+            ref = win[nm][h[2] + lo[2] - origin[2]:h[2] + hi[2] - origin[2],
+                          h[1] + lo[1] - origin[1]:h[1] + hi[1] - origin[1],
+                          h[0] + lo[0] - origin[0]:h[0] + hi[0] - origin[0]]
+            got = p.interior_view(p.tensors[nm])[lo[2]:hi[2], lo[1]:hi[1], lo[0]:hi[0]].cpu().numpy()
+            e = rel_err(got, ref)
+            assert e <= tolerance(prog["dtype"]), f"{workload} {nm} window {origin}: rel err {e}"

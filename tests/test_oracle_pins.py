@@ -428,3 +428,30 @@ def test_box_window_origin_translation():
     win = {k: np.ascontiguousarray(v[1:6, 0:7, 1:8]) for k, v in full.items()}
     OracleProgram(prog).run(win, n=(5, 5, 3), origin=(1, 0, 1))
     assert np.array_equal(win["O"][1:-1, 1:-1, 1:-1], ref["O"][2:5, 1:6, 2:7])
+
+
+@pytest.mark.parametrize("cfg", ["C5", "C3"])
+def test_window_evaluation_matches_full_grid(cfg):
+    """The sampled full-size GPU checks evaluate the oracle on w^3 windows with generated
+    ghosts; pinned here against the whole-grid oracle: exact inside the accumulated-reach
+    margin (and up to the global boundary on boundary sides)."""
+    import sys
+    sys.path.insert(0, os.path.dirname(os.path.abspath(__file__)))
+    from _harness import accumulated_reach, window_field
+    prog = {"C5": lambda: P.c5(nx=40, ny=36, nz=30), "C3": lambda: P.c3(nx=40, ny=36, nz=30)}[cfg]()
+    g = prog["grid"]
+    N, h = (g["nx"], g["ny"], g["nz"]), tuple(g["ghost"])
+    full = dense_arrays(prog, 4)
+    OracleProgram(prog).run(full)
+    m, w = accumulated_reach(prog), 24
+    for origin in [(0, 0, 0), tuple((N[d] - w) // 2 for d in range(3)), tuple(N[d] - w for d in range(3))]:
+        win = {a["name"]: window_field(4, aid, origin, (w, w, w), h, prog["dtype"])
+               for aid, a in enumerate(prog["arrays"])}
+        OracleProgram(prog).run(win, n=(w, w, w), origin=origin)
+        lo = [origin[d] + (m[d] if origin[d] > 0 else 0) for d in range(3)]
+        hi = [origin[d] + w - (m[d] if origin[d] + w < N[d] else 0) for d in range(3)]
+        for nm in [a["name"] for a in prog["arrays"] if a["role"] in ("out", "inout")]:
+            sl = lambda o: (slice(h[2] + lo[2] - o[2], h[2] + hi[2] - o[2]),  # noqa: E731
+                            slice(h[1] + lo[1] - o[1], h[1] + hi[1] - o[1]),
+                            slice(h[0] + lo[0] - o[0], h[0] + hi[0] - o[0]))
+            assert np.array_equal(win[nm][sl(origin)], full[nm][sl((0, 0, 0))]), (cfg, origin, nm)

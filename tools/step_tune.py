@@ -25,6 +25,10 @@ import bench  # noqa: E402
 from paper_conf_hpdc_wahibm15_b200 import Program, StencilError  # noqa: E402
 
 
+ZCHUNKS = ()          # () = the default rule (32 planes below 16 rows, else 16)
+PREFETCH = (2, 3)
+
+
 def candidates(ny):
     out = []
     for tx in (32, 64, 128):
@@ -37,9 +41,13 @@ def candidates(ny):
                 ty = nt // xt * by * cb
                 if ty > ny:
                     continue
-                for pf in (2, 3):
-                    out.append(dict(tile_x=tx, tile_y=ty, threads=nt, block_x=bx, block_y=by,
-                                    block_cby=cb, zchunk=32 if ty < 16 else 16, prefetch=pf))
+                # prefetch 1 frees ring planes for more resident CTAs; short chunks add
+                # warm-up planes but more CTAs (measured on C2: 32x16x8, prefetch 1 wins)
+                zcs = ZCHUNKS or ((32,) if ty < 16 else (16,))
+                for zc in zcs:
+                    for pf in PREFETCH:
+                        out.append(dict(tile_x=tx, tile_y=ty, threads=nt, block_x=bx, block_y=by,
+                                        block_cby=cb, zchunk=zc, prefetch=pf))
     return out
 
 
@@ -51,7 +59,12 @@ def main():
     ap.add_argument("--rounds", type=int, default=1)
     ap.add_argument("--steps", type=int, default=40)
     ap.add_argument("--groups", default=None, help="comma list of group indices (default all)")
+    ap.add_argument("--zchunks", default="", help="comma list of z-chunk lengths (default rule)")
+    ap.add_argument("--prefetch", default="2,3", help="comma list of prefetch depths")
     a = ap.parse_args()
+    global ZCHUNKS, PREFETCH
+    ZCHUNKS = tuple(int(v) for v in a.zchunks.split(",") if v)
+    PREFETCH = tuple(int(v) for v in a.prefetch.split(",") if v)
     prog = bench.load_workload(a.workload)
     plan = bench.plan_of(prog)
     cfgs = list(bench.tuned_configs(prog) or [None] * len(plan))

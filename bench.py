@@ -225,6 +225,29 @@ def run_ours(args):
     step_ms = s.elapsed_time(e) / args.steps
     clocks = sampler.stop()
     step_ms = max_over_ranks(step_ms)
+    # the same step captured once as a CUDA graph and replayed K times (SURVEY.md §8(d)
+    # timing protocol; S7): launch overhead off the host, same kernels
+    graph_ms = None
+    try:
+        g = torch.cuda.CUDAGraph()
+        gs = torch.cuda.Stream(device=dev)
+        gs.wait_stream(stream)
+        with torch.cuda.stream(gs):
+            with torch.cuda.graph(g, stream=gs):
+                p.run_fused(gs)
+        barrier()
+        g.replay()
+        s, e = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+        barrier()
+        s.record(stream)
+        for k in range(args.steps):
+            g.replay()
+        e.record(stream)
+        barrier()
+        graph_ms = max_over_ranks(s.elapsed_time(e) / args.steps)
+        del g
+    except Exception as ex:  # reported, never silently replacing the headline
+        graph_ms = f"capture failed: {ex}"
     # per-launch durations (dominant kernel of the roofline): a second timed pass of
     # the same launches with CUDA events between them on the launching stream
     prof_steps = max(3, min(args.steps, 50))
@@ -358,6 +381,8 @@ def run_ours(args):
             "e2e": {"value": updates / (e2e_ms * 1e-3), "unit": UNIT, "h2d_bytes_per_step": h2d,
                     "d2h_bytes_per_step": d2h, "ms_per_step": e2e_ms},
             # N > 1: a launch that receives ghost planes runs as interior + 2 boundary launches
+            "graph_replay": {"ms_per_step": graph_ms, "note": "one fused step captured as a CUDA "
+                             "graph, replayed K times (same kernels; not the headline)"},
             "gpu_launches": args.steps * sum(3 if world > 1 and p.exchange_plan("fused", i) else 1
                                              for i in live_f),
             "clocks": clocks,

@@ -243,3 +243,38 @@ def test_full_size_sampled_bench_configuration(cuda_device, workload, plan, w):
             got = p.interior_view(p.tensors[nm])[lo[2]:hi[2], lo[1]:hi[1], lo[0]:hi[0]].cpu().numpy()
             e = rel_err(got, ref)
             assert e <= tolerance(prog["dtype"]), f"{workload} {nm} window {origin}: rel err {e}"
+
+
+@pytest.mark.parametrize("mode", ["fused", "unfused"])
+def test_cuda_graph_capture_replay_bitexact(cuda_device, mode):
+    """S7: one step captured as a CUDA graph (torch.cuda.graph on its capture stream) and
+    replayed equals the eagerly launched step bit for bit; replays are idempotent."""
+    import sys
+    import torch
+    sys.path.insert(0, os.path.dirname(os.path.dirname(os.path.abspath(__file__))))
+    import bench
+    from _harness import gpu_program
+    prog = bench.load_workload("C4")
+    prog = dict(prog, grid=dict(prog["grid"], nx=256, nz=64))
+    p = gpu_program(prog, plan=prog["plans"]["fused"])
+    dev = torch.device("cuda:0")
+    p.allocate(dev, fill=0.0)
+    bench.fill_inputs(p, prog, dev, 0, prog["grid"]["ghost"][2])
+    outs = [a["name"] for a in prog["arrays"] if a["role"] in ("out", "inout")]
+    p.run(mode)  # loads modules and builds launch parameters outside the capture
+    torch.cuda.synchronize()
+    want = {n: p.interior_view(p.tensors[n]).clone() for n in outs}
+    for n in outs:
+        p.interior_view(p.tensors[n]).fill_(float("nan"))
+    g = torch.cuda.CUDAGraph()
+    s = torch.cuda.Stream(device=dev)
+    s.wait_stream(torch.cuda.current_stream())
+    with torch.cuda.stream(s):
+        with torch.cuda.graph(g, stream=s):
+            p.run(mode, s)
+    torch.cuda.synchronize()
+    for _ in range(3):
+        g.replay()
+    torch.cuda.synchronize()
+    for n in outs:
+        assert torch.equal(p.interior_view(p.tensors[n]), want[n]), f"{mode} {n}: graph replay differs"

@@ -29,6 +29,7 @@
 // array's ghost value through a predicated load; tiles inside the interior skip
 // the test.
 #include <cstdio>
+#include <cstdlib>
 #include <cstring>
 #include <functional>
 #include <set>
@@ -317,7 +318,7 @@ std::string generate_launch(const stencil_program *p, Launch &L, int index, bool
         // WAR: they have finished reading the ghosts this launch overwrites)
         o << "  sf_pdl_wait();\n";
         o << "  const unsigned long long xs_seq = sf_ld_volatile_u64(p.xs_self) + 1;\n";
-        if (std::getenv("SF_DEBUG_XP"))
+        if (std::getenv("SF_DEBUG_XP"))  // dev aid (tools/debug_xpush.py): per-CTA trace
             o << "  if (tid == 0) printf(\"[" << L.fn << "] own=%p seq=%llu Z0=%d zc=%d nlo=%d blk=%d,%d,%d\\n\", p.xs_own, xs_seq, Z0, zc, p.n_lo, blockIdx.x, blockIdx.y, blockIdx.z);\n";
         if (L.xp_dw > 0) {
             o << "  if (Z0 < " << L.xp_dw << " || Z0 + zc > NZ - " << L.xp_dw << ") {\n";

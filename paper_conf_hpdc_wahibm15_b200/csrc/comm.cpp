@@ -91,7 +91,6 @@ void exchange_schedule(const stencil_program *p, Mode &m) {
         L.xp = push && !L.dead;
         L.xp_dw = 0;
     }
-    const bool nowait = p->opt.xpush == 2;  // debugging only: the protocol without waits
     int first_live = -1;
     for (size_t i = 0; i < n && first_live < 0; ++i)
         if (!m.launches[i].dead) first_live = (int)i;
@@ -104,8 +103,8 @@ void exchange_schedule(const stencil_program *p, Mode &m) {
                 for (size_t s = 0; s < W.st.size(); ++s)
                     if (W.st[s].stored && W.st[s].out == a)
                         W.pushes.push_back({(int)s, above[a], below[a]});
-                if (!nowait) W.xp_dw = std::max({W.xp_dw, above[a], below[a]});
-                for (int r : (nowait ? std::vector<int>{} : readers[a])) {
+                W.xp_dw = std::max({W.xp_dw, above[a], below[a]});
+                for (int r : readers[a]) {
                     Launch &R = m.launches[r];
                     R.xp_dw = std::max({R.xp_dw, R.z_below, R.z_above});
                 }

@@ -259,6 +259,16 @@ sp_status fusion_plan_set(stencil_program *prog, int32_t n_groups, const int32_t
  * With group_begin == NULL only *n_groups is returned.  Does not set the plan. */
 sp_status sp_plan_greedy(stencil_program *prog, int32_t cap, int32_t *n_groups,
                          int32_t *group_begin, sp_stmt_ref *members);
+/* GGA-lite plan search (the paper's grouping genetic
+ * algorithm, whose encoding/operators are not in the paper): a
+ * grouping GA over fission units (statements may be grouped out of program order
+ * when independent), objective = the same launch-time model as sp_plan_greedy,
+ * illegal groupings (cyclic group order, R11 hazards, no tile fitting shared
+ * memory) rejected.  Seeded with the greedy plan, so its modelled cost is never
+ * worse.  Deterministic for (generations, population, seed).  Output as in
+ * sp_plan_greedy (call with group_begin == NULL first for *n_groups).  Host-only. */
+sp_status sp_plan_search(stencil_program *prog, int32_t generations, int32_t population, uint64_t seed,
+                         int32_t cap, int32_t *n_groups, int32_t *group_begin, sp_stmt_ref *members);
 
 /* mode 0 = unfused (one launch per original kernel), 1 = fused plan. */
 sp_status sp_plan_count(const stencil_program *prog, int32_t mode, int32_t *n_launches);

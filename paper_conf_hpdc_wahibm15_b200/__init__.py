@@ -307,6 +307,19 @@ class Program:
         return [[f"{names[mem[i].kernel]}:{mem[i].stmt}" for i in range(begin[g], begin[g + 1])]
                 for g in range(ng.value)]
 
+    def plan_search(self, generations=60, population=24, seed=1):
+        """GGA-lite fission/fusion plan search over the library's model (sp_plan_search)."""
+        ng = ctypes.c_int32()
+        args = (self.handle, int(generations), int(population), ctypes.c_uint64(seed))
+        _check(lib().sp_plan_search(*args, 0, ctypes.byref(ng), None, None))
+        nst = sum(len(k["stmts"]) for k in self.prog["kernels"])
+        begin = (ctypes.c_int32 * (ng.value + 1))()
+        mem = (SpStmtRef * nst)()
+        _check(lib().sp_plan_search(*args, ng.value, ctypes.byref(ng), begin, mem))
+        names = [k["name"] for k in self.prog["kernels"]]
+        return [[f"{names[mem[i].kernel]}:{mem[i].stmt}" for i in range(begin[g], begin[g + 1])]
+                for g in range(ng.value)]
+
     def n_launches(self, mode):
         n = ctypes.c_int32()
         _check(lib().sp_plan_count(self.handle, self._mode(mode), ctypes.byref(n)))

@@ -85,7 +85,7 @@ EXPORTS = [
     "sp_signal_buffer", "sp_bind_peer", "sp_bind_peer_signal", "sp_ipc_export", "sp_ipc_open", "stencil_program_create",
     "stencil_program_destroy", "stencil_program_layout", "stencil_program_bind",
     "sp_program_set_option", "sp_program_counts", "sp_program_edges", "sp_fission_components",
-    "fusion_plan_set", "sp_plan_greedy", "sp_plan_count", "sp_plan_report", "fusion_plan_report", "sp_plan_source",
+    "fusion_plan_set", "sp_plan_greedy", "sp_plan_search", "sp_plan_count", "sp_plan_report", "fusion_plan_report", "sp_plan_source",
     "sp_plan_exchange", "sp_plan_wave_offsets", "sp_plan_tune", "sp_compile", "sp_load", "run_unfused", "run_fused", "sp_run_launch", "exchange_halos", "sp_last_error",
 ]
 
@@ -120,6 +120,7 @@ def lib():
             "fusion_plan_set": [vp, i32, P(i32), P(SpStmtRef)],
             "sp_plan_count": [vp, i32, P(i32)],
             "sp_plan_greedy": [vp, i32, P(i32), P(i32), P(SpStmtRef)],
+            "sp_plan_search": [vp, i32, i32, ctypes.c_uint64, i32, P(i32), P(i32), P(SpStmtRef)],
             "sp_plan_report": [vp, i32, i32, P(SpGroupReport)],
             "fusion_plan_report": [vp, i32, P(SpGroupReport)],
             "sp_plan_source": [vp, i32, ctypes.c_char_p, ctypes.c_size_t, P(ctypes.c_size_t)],

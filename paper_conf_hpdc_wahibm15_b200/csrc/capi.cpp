@@ -434,23 +434,36 @@ sp_status fusion_plan_set(stencil_program *p, int32_t n_groups, const int32_t *g
     });
 }
 
+static void write_plan(const stencil_program *p, const std::vector<std::vector<int>> &gs, int32_t cap,
+                       int32_t *n_groups, int32_t *group_begin, sp_stmt_ref *members) {
+    *n_groups = (int)gs.size();
+    if (!group_begin || !members) return;
+    if (cap < (int)gs.size()) fail(SP_E_ARG, "group capacity too small");
+    int pos = 0;
+    group_begin[0] = 0;
+    for (size_t g = 0; g < gs.size(); ++g) {
+        for (int gid : gs[g]) {
+            const Stmt &S = p->stmts[gid];
+            members[pos++] = sp_stmt_ref{S.kernel, S.local};
+        }
+        group_begin[g + 1] = pos;
+    }
+}
+
 sp_status sp_plan_greedy(stencil_program *p, int32_t cap, int32_t *n_groups, int32_t *group_begin,
                          sp_stmt_ref *members) {
     return guard([&] {
         if (!p || !n_groups) fail(SP_E_ARG, "null argument");
-        std::vector<std::vector<int>> gs = greedy_plan(p);
-        *n_groups = (int)gs.size();
-        if (!group_begin || !members) return;
-        if (cap < (int)gs.size()) fail(SP_E_ARG, "group capacity too small");
-        int pos = 0;
-        group_begin[0] = 0;
-        for (size_t g = 0; g < gs.size(); ++g) {
-            for (int gid : gs[g]) {
-                const Stmt &S = p->stmts[gid];
-                members[pos++] = sp_stmt_ref{S.kernel, S.local};
-            }
-            group_begin[g + 1] = pos;
-        }
+        write_plan(p, greedy_plan(p), cap, n_groups, group_begin, members);
+    });
+}
+
+sp_status sp_plan_search(stencil_program *p, int32_t generations, int32_t population, uint64_t seed,
+                         int32_t cap, int32_t *n_groups, int32_t *group_begin, sp_stmt_ref *members) {
+    return guard([&] {
+        if (!p || !n_groups || generations < 0 || population < 1) fail(SP_E_ARG, "bad argument");
+        write_plan(p, search_plan(p, generations, population, seed), cap, n_groups, group_begin,
+                   members);
     });
 }
 

@@ -202,6 +202,8 @@ void analyze_mode(stencil_program *p, bool fused, const std::vector<std::vector<
                   Mode &out);
 void fill_report(const stencil_program *p, const Launch &L, sp_group_report *r);
 std::vector<std::vector<int>> greedy_plan(stencil_program *p);
+std::vector<std::vector<int>> search_plan(stencil_program *p, int generations, int population,
+                                          uint64_t seed);
 
 // codegen.cpp
 std::string generate_launch(const stencil_program *p, Launch &L, int index, bool fused);

@@ -278,3 +278,16 @@ def test_cuda_graph_capture_replay_bitexact(cuda_device, mode):
     torch.cuda.synchronize()
     for n in outs:
         assert torch.equal(p.interior_view(p.tensors[n]), want[n]), f"{mode} {n}: graph replay differs"
+
+
+@pytest.mark.parametrize("cfg", ["C3", "C4"])
+def test_ga_plan_parity_bitexact(cuda_device, cfg):
+    """Plans found by the GGA-lite search (sp_plan_search, NEXT #1) run bit-exact with
+    the oracle in the parity build (fmad=0), fused and unfused."""
+    from synth.scale_les import c4
+    from paper_conf_hpdc_wahibm15_b200 import Program
+    prog = {"C3": lambda: P.c3(nx=48, ny=20, nz=18), "C4": lambda: c4(nx=96, ny=32, nz=21)}[cfg]()
+    plan = Program(prog).plan_search(generations=20, population=12, seed=5)
+    ref = oracle_outputs(prog, seed=9)
+    got = gpu_run(prog, "fused", 9, options={"fmad": 0}, plan=plan)
+    assert_close(prog, got, ref, exact=True)

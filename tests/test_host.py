@@ -335,6 +335,50 @@ def test_greedy_plan_is_legal_and_reduces_traffic():
     assert len(refs) == len(set(refs)) == sum(len(k["stmts"]) for k in prog["kernels"])
 
 
+def _model_cost(p, plan):
+    p.set_plan(plan)
+    return sum(r["t_model_us"] for r in p.reports("fused"))
+
+
+@pytest.mark.parametrize("cfg", ["C3", "C4", "fuzz"])
+def test_ga_plan_search_legal_deterministic_not_worse(cfg):
+    """GGA-lite (sp_plan_search, NEXT #1): the plan is a legal partition accepted by
+    fusion_plan_set, identical for the same seed, and its modelled step time is not
+    above the greedy plan's (the GA is seeded with it; elitism)."""
+    import numpy as np
+    from synth.scale_les import c4
+    from _fuzz import random_lib_program
+    prog = {"C3": lambda: P.c3(n=64), "C4": lambda: c4(nx=256, ny=32, nz=64),
+            "fuzz": lambda: random_lib_program(np.random.default_rng(3))}[cfg]()
+    p = Program(prog)
+    g = p.plan_greedy()
+    s1 = p.plan_search(generations=25, population=12, seed=7)
+    assert s1 == p.plan_search(generations=25, population=12, seed=7)
+    refs = [r for grp in s1 for r in grp]
+    assert len(refs) == len(set(refs)) == sum(len(k["stmts"]) for k in prog["kernels"])
+    assert _model_cost(p, s1) <= _model_cost(p, g) * 1.02   # full vs quick tile search
+
+
+def test_ga_plan_search_interleaved_chains():
+    """Two independent chains interleaved in program order (A1, B1, A2, B2): the search
+    (whose decoding may group independent units out of program order) returns a legal
+    plan that moves each array once (no temp round trip)."""
+    T = P.tap
+    prog = {"name": "interleaved", "dtype": "f64", "grid": {"nx": 64, "ny": 32, "nz": 32, "ghost": [1, 1, 1]},
+            "arrays": [{"name": n, "role": r} for n, r in
+                       (("A", "in"), ("B", "in"), ("X", "temp"), ("Y", "temp"), ("OA", "out"), ("OB", "out"))],
+            "kernels": [P.kernel("A1", P.stmt("X", P.stencil_terms("A", P.PT7, [1 / 7] * 7))),
+                        P.kernel("B1", P.stmt("Y", P.stencil_terms("B", P.PT7, [1 / 7] * 7))),
+                        P.kernel("A2", P.stmt("OA", [{"c": 0.5, "a": T("X", (0, 0, 0))}])),
+                        P.kernel("B2", P.stmt("OB", [{"c": 0.5, "a": T("Y", (0, 0, 0))}]))]}
+    p = Program(prog)
+    s = p.plan_search(generations=30, population=16, seed=1)
+    p.set_plan(s)
+    assert _model_cost(p, s) <= _model_cost(p, p.plan_greedy()) * 1.02
+    fused = sum(r["bytes_alg"] for r in p.reports("fused"))
+    assert fused <= 4 * 8  # A, B, OA, OB once each
+
+
 def test_wave_offsets_raw_reach():
     """z-wave skew: K3 reads T2 one plane above (dz=+1), so it trails K2 by one plane;
     point-wise and in-plane reads need no skew."""

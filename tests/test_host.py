@@ -450,3 +450,29 @@ def test_box_validation_and_hazard():
     assert "R2'" in str(e.value)
     p.set_plan([["K0"], ["K1", "K2"]])                 # boxed writer alone in its group: fine
     p.compile("fused")
+
+
+def test_segment_dp_is_exact():
+    """The measured planner's segmentation DP (tools/plan_autotune.py, NEXT #1) returns
+    the optimum over contiguous segmentations, checked by brute force on random costs
+    (including illegal segments)."""
+    import itertools
+    import os
+    import sys
+    import numpy as np
+    sys.path.insert(0, os.path.join(os.path.dirname(os.path.dirname(os.path.abspath(__file__))), "tools"))
+    import importlib
+    pa = importlib.import_module("plan_autotune")
+    rng = np.random.default_rng(0)
+    for n, mu in ((6, 3), (7, 7), (8, 2)):
+        c = {(i, j): (float("inf") if rng.random() < 0.15 and j - i > 1 else float(rng.random() * (j - i) ** 0.7))
+             for i in range(n) for j in range(i + 1, n + 1)}
+        cuts = pa.segment_dp(n, lambda i, j: c[(i, j)], mu)
+        got = sum(c[(a, b)] for a, b in zip(cuts[:-1], cuts[1:]))
+        best = float("inf")
+        for mask in itertools.product([0, 1], repeat=n - 1):
+            cs = [0] + [i + 1 for i, m in enumerate(mask) if m] + [n]
+            if any(b - a > mu for a, b in zip(cs[:-1], cs[1:])):
+                continue
+            best = min(best, sum(c[(a, b)] for a, b in zip(cs[:-1], cs[1:])))
+        assert abs(got - best) < 1e-12 and all(b - a <= mu for a, b in zip(cuts[:-1], cuts[1:]))

@@ -173,6 +173,59 @@ def autotune(prog, log=print, max_group=64, hints=True):
     return groups, cost
 
 
+def fission_units(prog, full):
+    units = []
+    for k in prog["kernels"]:
+        comp, n = full.fission(k["name"])
+        pieces = [[] for _ in range(n)]
+        for i, c in enumerate(comp):
+            pieces[c].append(f"{k['name']}:{i}")
+        units += pieces
+    return units
+
+
+def dp_segment(prog, log=print, max_units=8, hints=True):
+    """Exact optimum over contiguous segmentations of the fission units (the space the
+    greedy merges walk) for the same measured objective (sum of isolated group times):
+    best[j] = min over i >= j - max_units of best[i] + t(units i..j-1).  Each segment
+    is timed once (cached)."""
+    T = Timer(prog)
+    if hints and prog["dtype"] == "f64":
+        T.hints = HINTS_F64
+    units = fission_units(prog, T._full)
+
+    def seg(i, j):
+        return T.time([r for u in units[i:j] for r in u])
+
+    cuts = segment_dp(len(units), seg, max_units,
+                      log=lambda j, b: log(f"prefix {j}/{len(units)}: {b*1e3:.3f} ms "
+                                           f"({len(T.cache)} segments timed)"))
+    groups = [[r for u in units[i:j] for r in u] for i, j in zip(cuts[:-1], cuts[1:])]
+    return groups, [T.time(g) for g in groups]
+
+
+def segment_dp(n, cost, max_units, log=None):
+    """Cut positions 0 = c0 < c1 < ... < ck = n minimising sum cost(c_i, c_i+1) over
+    segments of at most max_units units (cost inf: illegal segment)."""
+    inf = float("inf")
+    best = [0.0] + [inf] * n
+    arg = [0] * (n + 1)
+    for j in range(1, n + 1):
+        for i in range(max(0, j - max_units), j):
+            if best[i] == inf:
+                continue
+            t = cost(i, j)
+            if best[i] + t < best[j]:
+                best[j], arg[j] = best[i] + t, i
+        if log:
+            log(j, best[j])
+    cuts, j = [n], n
+    while j > 0:
+        j = arg[j]
+        cuts.insert(0, j)
+    return cuts
+
+
 def config_candidates(prog):
     ny = prog["grid"]["ny"]
     tiles = [32, 64] if prog["dtype"] == "f64" else [64, 128]
@@ -256,12 +309,16 @@ def main():
     ap.add_argument("--out", default=None)
     ap.add_argument("--tune", action="store_true", help="also tune each group's tile/block config")
     ap.add_argument("--plan-from", default=None, help="skip the search, tune this plan")
+    ap.add_argument("--dp", action="store_true", help="exact segmentation DP instead of greedy merges")
+    ap.add_argument("--max-units", type=int, default=8, help="DP: fission units per group at most")
     a = ap.parse_args()
     prog = bench.load_workload(a.workload)
     t0 = time.time()
     if a.plan_from:
         groups = json.load(open(a.plan_from))["groups"]
         cost = [0.0] * len(groups)
+    elif a.dp:
+        groups, cost = dp_segment(prog, log=lambda m: print(m, flush=True), max_units=a.max_units)
     else:
         groups, cost = autotune(prog, log=lambda m: print(m, flush=True))
     print(f"{len(groups)} groups, measured sum {sum(cost)*1e3:.3f} ms, search {time.time()-t0:.0f} s")
@@ -272,7 +329,8 @@ def main():
         p.set_plan(groups)
         fused = sum(r["bytes_alg"] for r in p.reports("fused")) / p.elem
         unfused = sum(r["bytes_alg"] for r in p.reports("unfused")) / p.elem
-        json.dump({"workload": a.workload, "planner": "measured greedy (tools/plan_autotune.py)",
+        planner = "measured segmentation DP" if a.dp else "measured greedy"
+        json.dump({"workload": a.workload, "planner": planner + " (tools/plan_autotune.py)",
                    "groups": groups, "group_ms": [c * 1e3 for c in cost], "configs": cfgs,
                    "passes": {"fused": fused, "unfused": unfused}}, open(a.out, "w"), indent=1)
         print("wrote", a.out)

@@ -228,8 +228,9 @@ std::string generate_launch(const stencil_program *p, Launch &L, int index, bool
     o << "  extern __shared__ __align__(128) unsigned char sf_smem[];\n";
     o << "  const int tid = threadIdx.x;\n";
     // chunks [0, n_lo) tile planes [z_base, z_mid), the others [z_hi, z_end)
-    if (L.xp)  // chunks next to the slab ends (which may wait for the neighbours) go last
-        o << "  const int bz = ((int)blockIdx.z + 1) % (int)gridDim.z, lo = bz < p.n_lo;\n";
+    if (L.xp)  // the slab's end chunks go first (order 0, last, 1, 2, ...): they carry the
+               // neighbour exchange, and signal it as soon as they are done
+        o << "  const int bz = sf_xs_chunk((int)blockIdx.z, (int)gridDim.z), lo = bz < p.n_lo;\n";
     else
         o << "  const int bz = (int)blockIdx.z, lo = bz < p.n_lo;\n";
     o << "  const int X0 = (int)blockIdx.x * TX, Y0 = (int)blockIdx.y * TY,\n"
@@ -312,17 +313,20 @@ std::string generate_launch(const stencil_program *p, Launch &L, int index, bool
     o << "  }\n  __syncthreads();\n";
     if (L.xp) {
         // peer-push protocol: this kernel is number seq of
-        // the rank's launches; a chunk within xp_dw planes of a slab end reads ghost
-        // planes the neighbours push, or pushes into theirs, so it first waits until
-        // both neighbours have completed launch seq-1 (RAW: their pushes are visible;
-        // WAR: they have finished reading the ghosts this launch overwrites)
+        // the rank's launches; a chunk within xp_dw planes of the bottom (top) slab end
+        // reads ghost planes the lower (upper) neighbour pushes, or pushes into its
+        // ghosts, so it first waits until that neighbour's end chunks facing this rank
+        // have completed launch seq-1 (RAW: their pushes are visible; WAR: they have
+        // finished reading the ghosts this launch overwrites)
         o << "  sf_pdl_wait();\n";
         o << "  const unsigned long long xs_seq = sf_ld_volatile_u64(p.xs_self) + 1;\n";
         if (std::getenv("SF_DEBUG_XP"))  // dev aid (tools/debug_xpush.py): per-CTA trace
             o << "  if (tid == 0) printf(\"[" << L.fn << "] own=%p seq=%llu Z0=%d zc=%d nlo=%d blk=%d,%d,%d\\n\", p.xs_own, xs_seq, Z0, zc, p.n_lo, blockIdx.x, blockIdx.y, blockIdx.z);\n";
-        if (L.xp_dw > 0) {
-            o << "  if (Z0 < " << L.xp_dw << " || Z0 + zc > NZ - " << L.xp_dw << ") {\n";
-            o << "    if (tid == 0) sf_xs_wait(p.xs_own, p.xs_dn != nullptr, p.xs_up != nullptr, xs_seq - 1);\n";
+        const int DW = L.xp_dw;
+        o << "  const bool xs_bot = Z0 < " << DW << ", xs_top = Z0 + zc > NZ - " << DW << ";\n";
+        if (DW > 0) {
+            o << "  if (xs_bot || xs_top) {\n";
+            o << "    if (tid == 0) sf_xs_wait(p.xs_own, xs_bot && p.xs_dn, xs_top && p.xs_up, xs_seq - 1);\n";
             o << "    __syncthreads();\n  }\n";
         }
     }
@@ -913,10 +917,28 @@ std::string generate_launch(const stencil_program *p, Launch &L, int index, bool
     o << "  }\n";
     if (L.xp) {
         // completion: the last CTA publishes seq to itself and to both neighbours
-        o << "  __threadfence_system();  // this thread's stores (incl. peer pushes) first\n";
-        o << "  sf_bar_sync(3, NT);\n";
+        // only the end chunks push or read pushed planes: they alone fence at system
+        // scope before their CTA's completion (a middle chunk's stores are ordered for
+        // this rank's next launch by stream order)
+        o << "  if (xs_bot || xs_top) {\n";
+        o << "    __threadfence_system();  // this thread's stores (incl. peer pushes) first\n";
+        o << "    sf_bar_sync(3, NT);\n  }\n";
         if (std::getenv("SF_DEBUG_XP"))
             o << "  if (tid == 0) printf(\"[" << L.fn << "] own=%p seq=%llu Z0=%d done\\n\", p.xs_own, xs_seq, Z0);\n";
+        if (L.xp_dw > 0) {
+            // the end chunks facing a neighbour publish to it as soon as they are all done
+            o << "  if (tid == 0 && (xs_bot || xs_top)) {\n";
+            o << "    int nb = 0, nt = 0;  // end chunks of this launch, per side\n";
+            o << "    for (int c = 0; c < (int)gridDim.z; ++c) {\n";
+            o << "      const int l = c < p.n_lo, z0 = l ? p.z_base + c * ZC : p.z_hi + (c - p.n_lo) * ZC;\n";
+            o << "      const int n = min(ZC, (l ? p.z_mid : p.z_end) - z0);\n";
+            o << "      nb += z0 < " << L.xp_dw << "; nt += z0 + n > NZ - " << L.xp_dw << ";\n";
+            o << "    }\n";
+            o << "    const unsigned per = gridDim.x * gridDim.y;\n";
+            o << "    if (xs_bot && p.xs_dn) sf_xs_signal_side((unsigned *)(p.xs_own + 3) + 1, per * nb, p.xs_dn + 1, xs_seq);\n";
+            o << "    if (xs_top && p.xs_up) sf_xs_signal_side((unsigned *)(p.xs_own + 4), per * nt, p.xs_up + 0, xs_seq);\n";
+            o << "  }\n";
+        }
         o << "  if (tid == 0) sf_xs_signal(p.xs_ctr, gridDim.x * gridDim.y * gridDim.z, p.xs_self, "
              "p.xs_dn, p.xs_up, xs_seq);\n";
     }

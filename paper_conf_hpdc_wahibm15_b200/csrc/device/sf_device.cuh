@@ -153,7 +153,8 @@ __device__ __forceinline__ float sf_ld(const float *p) {
 // ---- peer-push halo protocol (several ranks, option xpush) --------------------
 // Signal block of a rank (64 B, device memory of that rank, mapped by its
 // neighbours): u64 [0] progress published by the lower neighbour, [1] by the
-// upper neighbour, [2] this rank's own progress; u32 at byte 24: CTAs done.
+// upper neighbour, [2] this rank's own progress; u32 at byte 24: CTAs done,
+// byte 28: bottom end CTAs done, byte 32: top end CTAs done.
 __device__ __forceinline__ sf_u64 sf_ld_volatile_u64(const sf_u64 *p) {
     sf_u64 v;
     asm volatile("ld.volatile.global.u64 %0, [%1];" : "=l"(v) : "l"(p) : "memory");
@@ -182,6 +183,20 @@ __device__ __forceinline__ void sf_xs_wait(const sf_u64 *own, bool has_dn, bool 
     }
     // the pushed planes were written through the generic proxy; TMA reads them
     asm volatile("fence.proxy.async.global;" ::: "memory");
+}
+// order of the chunks: the two slab-end chunks first (0, last), then the middle
+__device__ __forceinline__ int sf_xs_chunk(int b, int n) {
+    return n < 2 || b == 0 ? b : (b == 1 ? n - 1 : b - 1);
+}
+// end-chunk completion of one side: the last of its `total` CTAs publishes seq into
+// the neighbour's slot (the whole-grid signal below publishes it again, harmlessly)
+__device__ __forceinline__ void sf_xs_signal_side(sf_u32 *ctr, sf_u32 total, sf_u64 *slot, sf_u64 seq) {
+    sf_u32 old;
+    asm volatile("atom.acq_rel.gpu.global.add.u32 %0, [%1], 1;" : "=r"(old) : "l"(ctr) : "memory");
+    if (old != total - 1) return;
+    asm volatile("st.relaxed.gpu.global.u32 [%0], 0;" ::"l"(ctr) : "memory");
+    asm volatile("fence.sc.sys;" ::: "memory");
+    sf_st_release_sys(slot, seq);
 }
 // CTA completion; the last CTA of the grid publishes seq (own progress and both
 // neighbours' "from" slots) after a system-scope fence

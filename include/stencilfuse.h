@@ -224,6 +224,11 @@ sp_status stencil_program_bind(stencil_program *prog, int32_t array, void *dev_p
  *   "pdl"       0|1|2 programmatic dependent launch: off / fused groups / all
  *   "zwave"     S > 0: fused mode runs the z-wave schedule (sp_plan_wave_offsets)
  *   "zwave_streams" 1..8 waves in flight for "zwave" (default 2)
+ *   "xpush"     1: peer-push halo exchange of TEMP epochs on several ranks (see
+ *               sp_bind_peer); 0 (default): the communicator carries every epoch
+ *   "regcap"    occupancy-aware register cap at JIT time (recompile with
+ *               __maxnreg__ when a few registers cost a resident CTA, kept only
+ *               without spills): 0 never, 1 peer-push kernels (default), 2 all
  *   "suspend_hint", "coef_const", "l2pf", "acc_split"   measured-off experiments
  *   "num_sms"   SM count assumed by the tile chooser (default 148)
  *   "l2_flush"  unused by the library (reserved) */

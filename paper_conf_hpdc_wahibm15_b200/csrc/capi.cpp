@@ -379,6 +379,7 @@ sp_status sp_program_set_option(stencil_program *p, const char *key, int64_t v) 
         else if (k == "zwave") o.zwave = (int)v;
         else if (k == "zwave_streams") o.zwave_streams = std::max(1, std::min(8, (int)v));
         else if (k == "xpush") o.xpush = v != 0;
+        else if (k == "regcap") o.regcap = (int)std::min<int64_t>(v, 2);
         else if (k == "l2_flush") {}
         else fail(SP_E_ARG, "unknown option '" + k + "'");
         if (v < 0 && k != "prefetch") fail(SP_E_ARG, "negative option value");

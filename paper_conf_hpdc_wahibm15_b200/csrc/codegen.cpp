@@ -228,8 +228,8 @@ std::string generate_launch(const stencil_program *p, Launch &L, int index, bool
     o << "  extern __shared__ __align__(128) unsigned char sf_smem[];\n";
     o << "  const int tid = threadIdx.x;\n";
     // chunks [0, n_lo) tile planes [z_base, z_mid), the others [z_hi, z_end)
-    if (L.xp)  // the slab's end chunks go first (order 0, last, 1, 2, ...): they carry the
-               // neighbour exchange, and signal it as soon as they are done
+    if (L.xp && L.xp_dw > 0)  // the slab's end chunks go first (order 0, last, 1, 2, ...): they
+                              // carry the neighbour exchange, and signal it as soon as done
         o << "  const int bz = sf_xs_chunk((int)blockIdx.z, (int)gridDim.z), lo = bz < p.n_lo;\n";
     else
         o << "  const int bz = (int)blockIdx.z, lo = bz < p.n_lo;\n";
@@ -319,7 +319,9 @@ std::string generate_launch(const stencil_program *p, Launch &L, int index, bool
         // have completed launch seq-1 (RAW: their pushes are visible; WAR: they have
         // finished reading the ghosts this launch overwrites)
         o << "  sf_pdl_wait();\n";
-        o << "  const unsigned long long xs_seq = sf_ld_volatile_u64(p.xs_self) + 1;\n";
+        // only thread 0 waits and publishes: one load of the counter per CTA (every
+        // thread loading the same word would serialise on one L2 slice)
+        o << "  const unsigned long long xs_seq = tid == 0 ? sf_ld_volatile_u64(p.xs_self) + 1 : 0;\n";
         if (std::getenv("SF_DEBUG_XP"))  // dev aid (tools/debug_xpush.py): per-CTA trace
             o << "  if (tid == 0) printf(\"[" << L.fn << "] own=%p seq=%llu Z0=%d zc=%d nlo=%d blk=%d,%d,%d\\n\", p.xs_own, xs_seq, Z0, zc, p.n_lo, blockIdx.x, blockIdx.y, blockIdx.z);\n";
         const int DW = L.xp_dw;
@@ -922,7 +924,7 @@ std::string generate_launch(const stencil_program *p, Launch &L, int index, bool
         // this rank's next launch by stream order)
         o << "  if (xs_bot || xs_top) {\n";
         o << "    __threadfence_system();  // this thread's stores (incl. peer pushes) first\n";
-        o << "    sf_bar_sync(3, NT);\n  }\n";
+        o << "    sf_bar_sync(1, NT);  // the compute threads' barrier (ptxas: no extra barrier)\n  }\n";
         if (std::getenv("SF_DEBUG_XP"))
             o << "  if (tid == 0) printf(\"[" << L.fn << "] own=%p seq=%llu Z0=%d done\\n\", p.xs_own, xs_seq, Z0);\n";
         if (L.xp_dw > 0) {

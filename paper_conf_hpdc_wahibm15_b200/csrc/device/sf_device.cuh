@@ -190,9 +190,15 @@ __device__ __forceinline__ int sf_xs_chunk(int b, int n) {
 }
 // end-chunk completion of one side: the last of its `total` CTAs publishes seq into
 // the neighbour's slot (the whole-grid signal below publishes it again, harmlessly)
+// The counters use relaxed atomics: a CTA whose stores a neighbour depends on (an
+// end chunk) executed fence.sc.sys (__threadfence_system) before its increment, and
+// the last CTA executes fence.sc.sys before publishing, which orders those stores
+// before the publication (fence-fence synchronisation through the atomic's RMW
+// chain).  A release atomic in every CTA would stall each exiting CTA's SM on a
+// gpu-scope membar (measured: 23 % on a C5 group).
 __device__ __forceinline__ void sf_xs_signal_side(sf_u32 *ctr, sf_u32 total, sf_u64 *slot, sf_u64 seq) {
     sf_u32 old;
-    asm volatile("atom.acq_rel.gpu.global.add.u32 %0, [%1], 1;" : "=r"(old) : "l"(ctr) : "memory");
+    asm volatile("atom.relaxed.gpu.global.add.u32 %0, [%1], 1;" : "=r"(old) : "l"(ctr) : "memory");
     if (old != total - 1) return;
     asm volatile("st.relaxed.gpu.global.u32 [%0], 0;" ::"l"(ctr) : "memory");
     asm volatile("fence.sc.sys;" ::: "memory");
@@ -203,7 +209,7 @@ __device__ __forceinline__ void sf_xs_signal_side(sf_u32 *ctr, sf_u32 total, sf_
 __device__ __forceinline__ void sf_xs_signal(sf_u32 *ctr, sf_u32 total, sf_u64 *self, sf_u64 *dn,
                                              sf_u64 *up, sf_u64 seq) {
     sf_u32 old;
-    asm volatile("atom.acq_rel.gpu.global.add.u32 %0, [%1], 1;" : "=r"(old) : "l"(ctr) : "memory");
+    asm volatile("atom.relaxed.gpu.global.add.u32 %0, [%1], 1;" : "=r"(old) : "l"(ctr) : "memory");
     if (old != total - 1) return;
     asm volatile("st.relaxed.gpu.global.u32 [%0], 0;" ::"l"(ctr) : "memory");
     asm volatile("fence.sc.sys;" ::: "memory");

@@ -104,16 +104,18 @@ bool driver_mem_range(CUdeviceptr *base, size_t *size, CUdeviceptr p) {
 // ------------------------------------------------------------------ NVRTC
 static std::mutex g_cache_mu;
 static std::unordered_map<std::string, std::pair<std::string, int>> g_cache;  // key -> (cubin, regs)
+static std::unordered_map<std::string, int> g_spill;  // key -> spill store bytes
 
 static std::string compile_one(const std::string &src, bool fmad, const std::string &name,
-                               int *regs) {
+                               int *regs, int maxrreg = 0, int *spill_out = nullptr) {
     std::string key = std::to_string(std::hash<std::string>{}(src)) + (fmad ? "f" : "n") +
-                      std::to_string(src.size());
+                      std::to_string(src.size()) + "r" + std::to_string(maxrreg);
     {
         std::lock_guard<std::mutex> lk(g_cache_mu);
         auto it = g_cache.find(key);
         if (it != g_cache.end()) {
             *regs = it->second.second;
+            if (spill_out) *spill_out = g_spill[key];
             return it->second.first;
         }
     }
@@ -127,6 +129,8 @@ static std::string compile_one(const std::string &src, bool fmad, const std::str
                                       fmad ? "--fmad=true" : "--fmad=false", "--ftz=false",
                                       "--prec-div=true", "--prec-sqrt=true",
                                       "--ptxas-options=-v", "-DNDEBUG"};
+    const std::string mr = "--maxrregcount=" + std::to_string(maxrreg);
+    if (maxrreg > 0) opts.push_back(mr.c_str());
     nvrtcResult r = nvrtcCompileProgram(prog, (int)opts.size(), opts.data());
     size_t log_size = 0;
     nvrtcGetProgramLogSize(prog, &log_size);
@@ -144,14 +148,16 @@ static std::string compile_one(const std::string &src, bool fmad, const std::str
     int rr = -1;
     auto pos = log.find("Used ");
     if (pos != std::string::npos) rr = std::atoi(log.c_str() + pos + 5);
+    int spill = 0;
     if (log.find("bytes spill stores") != std::string::npos) {
         auto sp = log.find("bytes spill stores");
         auto b = log.rfind(',', sp);
-        int spill = std::atoi(log.c_str() + (b == std::string::npos ? 0 : b + 1));
-        if (spill > 0) std::fprintf(stderr, "[stencilfuse] warning: %s spills %d bytes\n",
-                                    name.c_str(), spill);
+        spill = std::atoi(log.c_str() + (b == std::string::npos ? 0 : b + 1));
+        if (spill > 0 && maxrreg == 0)
+            std::fprintf(stderr, "[stencilfuse] warning: %s spills %d bytes\n", name.c_str(), spill);
     }
     *regs = rr;
+    if (spill_out) *spill_out = spill;
     if (const char *dir = std::getenv("SF_DUMP_DIR")) {  // debugging aid: source, cubin, log
         std::string base = std::string(dir) + "/" + name;
         if (FILE *f = std::fopen((base + ".cu").c_str(), "w")) { std::fwrite(src.data(), 1, src.size(), f); std::fclose(f); }
@@ -160,7 +166,32 @@ static std::string compile_one(const std::string &src, bool fmad, const std::str
     }
     std::lock_guard<std::mutex> lk(g_cache_mu);
     g_cache[key] = {cubin, rr};
+    g_spill[key] = spill;
     return cubin;
+}
+
+// Resident CTAs per SM of a launch as the hardware allocates them: registers per
+// warp in units of 256, each of the 4 SM sub-partitions holding 16K registers and
+// a quarter of the resident warps (ceil); shared memory 228 KB with 1 KB reserved
+// per CTA; at most 64 warps and 32 CTAs.  Measured on B200 (ncu occupancy limits):
+// 160-thread CTAs fit 3 per SM at 128 registers and 2 at 132.
+static int resident_ctas(int regs, int nth, int64_t smem, int *by_regs, int *by_rest) {
+    const int w = (nth + 31) / 32;
+    int rest = std::min<int64_t>({32, 64 / w, (228 * 1024) / (smem + 1024)});
+    int rr = 0;
+    const int rw = (std::max(regs, 1) * 32 + 255) / 256 * 256;
+    for (int c = 1; c <= 32; ++c)
+        if (((c * w + 3) / 4) * rw <= 16384) rr = c;
+    if (by_regs) *by_regs = rr;
+    if (by_rest) *by_rest = rest;
+    return std::min(rr, rest);
+}
+
+// largest register count that keeps `target` CTAs of nth threads resident
+static int regs_for_ctas(int target, int nth) {
+    const int w = (nth + 31) / 32;
+    const int per_part = (target * w + 3) / 4;
+    return std::min(255, 16384 / per_part / 256 * 256 / 32);
 }
 
 void compile_mode(stencil_program *p, Mode &m) {
@@ -176,6 +207,34 @@ void compile_mode(stencil_program *p, Mode &m) {
             if (L.dead) continue;
             try {
                 L.cubin = compile_one(L.source, p->opt.fmad != 0, L.fn, &L.regs);
+                // occupancy-aware register cap: when the kernel sits a few registers
+                // above the budget of one more resident CTA that shared memory would
+                // allow, recompile at that budget and keep it if ptxas needs no spills.
+                // Default (1): peer-push kernels only, whose protocol adds a few
+                // registers to a tuned kernel (C5: 128 -> 132 regs cost a resident CTA
+                // and 23 %; capped: 114 regs, back to 3 CTAs/SM); 2: every kernel
+                // (measured on the single-GPU C4 step: 1 % slower, so not default)
+                int by_regs = 0, by_rest = 0;
+                resident_ctas(L.regs, L.nth, L.smem, &by_regs, &by_rest);
+                const bool capit = p->opt.regcap == 2 || (p->opt.regcap == 1 && L.xp);
+                if (capit && by_regs < by_rest) {
+                    const int cap = regs_for_ctas(by_regs + 1, L.nth);
+                    if (cap >= 32 && L.regs - cap <= 16) {
+                        int r2 = 0, spill = 0;
+                        // __launch_bounds__ overrides --maxrregcount and ptxas does not
+                        // model the per-sub-partition limit: state the budget directly
+                        std::string src2 = L.source;
+                        const std::string lb = "__launch_bounds__(" + std::to_string(L.nth) + ", 1)";
+                        const size_t at = src2.find(lb);
+                        if (at != std::string::npos)
+                            src2.replace(at, lb.size(), "__maxnreg__(" + std::to_string(cap) + ")");
+                        std::string c2 = compile_one(src2, p->opt.fmad != 0, L.fn, &r2, 0, &spill);
+                        if (spill == 0 && r2 > 0 && r2 <= cap) {
+                            L.cubin = c2;
+                            L.regs = r2;
+                        }
+                    }
+                }
             } catch (const Error &e) {
                 errs[i] = e.msg;
             }

@@ -25,7 +25,7 @@ ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
 sys.path.insert(0, ROOT)
 
 
-def worker(rank, world, port, workload, steps, q):
+def worker(rank, world, port, workload, steps, q, independent=False, xpush=1):
     sys.path.insert(0, ROOT)
     import torch
     import torch.distributed as dist
@@ -47,18 +47,23 @@ def worker(rank, world, port, workload, steps, q):
         zhalo = max([max(r["z_below"], r["z_above"]) for m in ("fused", "unfused")
                      for r in probe.reports(m)] + [loc["grid"]["ghost"][2]])
         comm = Comm.loopback(world)[rank]  # rank count only; no run_fused transport here
-        p = Program(loc, comm=comm, nz_global=nz * world, z_offset=rank * nz, zhalo=zhalo,
-                    options={"xpush": 1})
+        if independent:  # baseline: the same slabs as unrelated single-domain problems
+            p = Program(loc)
+            zhalo = loc["grid"]["ghost"][2]
+        else:
+            p = Program(loc, comm=comm, nz_global=nz * world, z_offset=rank * nz, zhalo=zhalo,
+                        options={"xpush": xpush})
         p.set_plan(plan)
         bench.apply_tuning(p, prog)
         p.allocate(dev, fill=0.0)
         bench.fill_inputs(p, loc, dev, rank * nz, zhalo)
         p.load("fused")
-        p.connect_peers(rank, world)
+        if not independent and xpush:
+            p.connect_peers(rank, world)
         oz = p.layout["origin_z"]
         n = p.n_launches("fused")
-        x0 = p.exchange_plan("fused", 0)
-        assert all(not p.exchange_plan("fused", i) for i in range(1, n))
+        x0 = [] if independent else p.exchange_plan("fused", 0)
+        assert independent or all(not p.exchange_plan("fused", i) for i in range(1, n))
         times = []
         for step in range(steps + 2):
             torch.cuda.synchronize()
@@ -113,7 +118,7 @@ def worker(rank, world, port, workload, steps, q):
                 if step >= 2:
                     ts.append(s.elapsed_time(e))
             res["ms_per_step_single"] = sorted(ts)[len(ts) // 2]
-            res["bitexact"] = all(torch.equal(torch.cat([g[nm] for g in got], dim=0),
+            res["bitexact"] = independent or all(torch.equal(torch.cat([g[nm] for g in got], dim=0),
                                               single.interior_view(single.tensors[nm]).cpu())
                                   for nm in outs)
         q.put((rank, res))
@@ -130,6 +135,10 @@ def main():
     ap.add_argument("--ranks", type=int, default=2)
     ap.add_argument("--steps", type=int, default=10)
     ap.add_argument("--no-mps", action="store_true")
+    ap.add_argument("--xpush", type=int, default=1, help="0: plain multi-rank kernels (valid only "
+                    "when every exchange is a step-start one, e.g. C5)")
+    ap.add_argument("--independent", action="store_true",
+                    help="baseline: the slabs as unrelated problems (no protocol, no exchange)")
     a = ap.parse_args()
     env = dict(os.environ)
     tmp = tempfile.mkdtemp(prefix="sf_mps_")
@@ -148,7 +157,7 @@ def main():
         sk.close()
         ctx = mp.get_context("spawn")
         q = ctx.Queue()
-        ps = [ctx.Process(target=worker, args=(r, a.ranks, port, a.workload, a.steps, q))
+        ps = [ctx.Process(target=worker, args=(r, a.ranks, port, a.workload, a.steps, q, a.independent, a.xpush))
               for r in range(a.ranks)]
         for p in ps:
             p.start()
@@ -159,7 +168,7 @@ def main():
         if isinstance(r0, str):
             print(r0)
             sys.exit(1)
-        r0.update(workload=a.workload, ranks=a.ranks, mps=not a.no_mps,
+        r0.update(workload=a.workload, ranks=a.ranks, mps=not a.no_mps, independent=a.independent, xpush=a.xpush,
                   overhead=r0["ms_per_step_ranks"] / r0["ms_per_step_single"] - 1)
         print(json.dumps(r0), flush=True)
     finally:

@@ -435,9 +435,15 @@ static void choose_config(const stencil_program *p, Launch &L, bool quick = fals
                                 C.nty = (int)((g.ny + ty - 1) / ty);
                                 C.nch = (int)((nz + C.zc - 1) / C.zc);
                                 double ctas = (double)C.ntx * C.nty * C.nch;
+                                // registers: per warp in units of 256, each of the 4 SM
+                                // sub-partitions holds 16K and a quarter of the warps
+                                const int wpc = (C.nth + 31) / 32, rw = regs_alloc * 32 / 256 * 256;
+                                int by_regs = 0;
+                                for (int c = 1; c <= 32; ++c)
+                                    if (((c * wpc + 3) / 4) * rw <= 16384) by_regs = c;
                                 int per_sm = (int)std::min<int64_t>(
                                     {(int64_t)(228 * 1024 / (C.smem + 1024)), (int64_t)(2048 / C.nth),
-                                     32, (int64_t)(65536 / (C.nth * regs_alloc))});
+                                     32, (int64_t)by_regs});
                                 if (per_sm < 1) continue;
                                 // Launch-time model, fitted to measured sweeps of C2/C3/C4/C5
                                 // groups (tools/model_fit.py, profiles/sweeps/): the busiest

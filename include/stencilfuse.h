@@ -229,7 +229,9 @@ sp_status stencil_program_bind(stencil_program *prog, int32_t array, void *dev_p
  *   "regcap"    occupancy-aware register cap at JIT time (recompile with
  *               __maxnreg__ when a few registers cost a resident CTA, kept only
  *               without spills): 0 never, 1 peer-push kernels (default), 2 all
- *   "suspend_hint", "coef_const", "l2pf", "acc_split"   measured-off experiments
+ *   "l2pf"      TMA L2 prefetch of input planes this many steps beyond the
+ *               shared-memory ring (default 1; 0 off)
+ *   "suspend_hint", "coef_const", "acc_split"   measured-off experiments
  *   "num_sms"   SM count assumed by the tile chooser (default 148)
  *   "l2_flush"  unused by the library (reserved) */
 sp_status sp_program_set_option(stencil_program *prog, const char *key, int64_t value);

@@ -37,7 +37,8 @@ struct Options {
     int block_x = 0, block_y = 0, block_cby = 0;  // register-block overrides (0 = chooser)
     int zqueue = 0;  // z-queues cost registers/occupancy more than they save (measured r1)
     int suspend_hint = 0;  // ns hint of mbarrier.try_wait (0 = none)
-    int l2pf = 0;          // TMA L2 prefetch distance in steps beyond the ring (0 = off)
+    int l2pf = 1;          // TMA L2 prefetch distance in steps beyond the ring (0 = off;
+                           // r1s3: 1 wins with the prefetch-1 rings: C2 -3.4 %, C5 -2 %, C4 -0.7 %)
     int coef_const = 0;    // 1: coefficients in a __constant__ table (r1: 35 % slower)
     int pdl = 1;        // programmatic dependent launch: 1 = fused groups, 2 = all, 0 = off
     int acc_split = 1;  // >1: interleaved partial sums in the perf build (no gain measured r1)

@@ -16,8 +16,9 @@ base = None
 for spec in sys.argv[2:]:
     opts = {kv.split("=")[0]: int(kv.split("=")[1]) for kv in spec.split(",") if kv}
     p = Program(prog, options=opts)
-    p.set_plan(bench.plan_of(prog))
-    bench.apply_tuning(p, prog)
+    plan = os.environ.get("SF_PLAN", "fused")
+    p.set_plan(bench.plan_of(prog, plan))
+    bench.apply_tuning(p, prog, plan)
     if base is None:
         p.allocate(dev, fill=0.0)
         bench.fill_inputs(p, prog, dev, 0, prog["grid"]["ghost"][2])

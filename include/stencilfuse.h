@@ -308,10 +308,13 @@ sp_status sp_plan_tune(stencil_program *prog, int32_t mode, int32_t launch, cons
  * arrays[], *n = total), with the planes received into the bottom ghost
  * (below[i]) and the top ghost (above[i]); below/above may be NULL.  An array
  * is received once per epoch (step start, or a launch that stores it, up to the
- * next), before the epoch's first launch that reads it beyond the slab, at the
- * largest depth any reader of the epoch needs (each <= zhalo).  run_unfused /
- * run_fused perform exactly this exchange, overlapped with the launch's
- * interior planes; host-only (no GPU needed). */
+ * next), at the largest depth any reader of the epoch needs (each <= zhalo):
+ * an epoch that begins at a store before its first launch that reads the array
+ * beyond the slab, every step-start epoch in one exchange before the step's
+ * first launch.  With option "xpush" the epochs of TEMP arrays that begin at a
+ * store are pushed by the storing kernel instead and do not appear here.
+ * run_unfused / run_fused perform exactly this exchange, overlapped with the
+ * launch's interior planes; host-only (no GPU needed). */
 sp_status sp_plan_exchange(stencil_program *prog, int32_t mode, int32_t launch, int32_t cap,
                            int32_t *arrays, int32_t *below, int32_t *above, int32_t *n);
 /* z-wave schedule of the fused mode (options "zwave" = S planes per wave,

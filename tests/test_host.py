@@ -476,3 +476,34 @@ def test_segment_dp_is_exact():
                 continue
             best = min(best, sum(c[(a, b)] for a, b in zip(cs[:-1], cs[1:])))
         assert abs(got - best) < 1e-12 and all(b - a <= mu for a, b in zip(cuts[:-1], cuts[1:]))
+
+
+@pytest.mark.parametrize("mode", ["fused", "unfused"])
+def test_peer_push_schedule_and_codegen(mode):
+    """NEXT #2 host side (no GPU): with option xpush on a 2-rank communicator, every TEMP
+    epoch that begins at a store leaves the communicator's schedule (its storing kernel
+    pushes it), step-start epochs stay, the generated kernels carry the push stores and
+    the progress protocol, and they compile for sm_100a (NVRTC)."""
+    from synth.scale_les import c4
+    from paper_conf_hpdc_wahibm15_b200 import Comm
+    import json
+    import os
+    prog = c4(nx=64, ny=32, nz=16)
+    root = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+    prog["plans"]["fused"] = json.load(open(os.path.join(root, "configs", "c4_plan.json")))["groups"]
+    temps = {a["name"] for a in prog["arrays"] if a["role"] == "temp"}
+    comms = Comm.loopback(2)
+    p = Program(prog, comm=comms[0], nz_global=32, z_offset=0, zhalo=4, options={"xpush": 1})
+    q = Program(prog, comm=comms[1], nz_global=32, z_offset=16, zhalo=4)
+    for x in (p, q):
+        x.set_plan(prog["plans"]["fused"])
+    n = p.n_launches(mode)
+    with_push = [p.exchange_plan(mode, i) for i in range(n)]
+    without = [q.exchange_plan(mode, i) for i in range(n)]
+    assert not any(a in temps for x in with_push for a, _, _ in x)
+    assert with_push[0] == without[0]                       # step-start epochs unchanged
+    assert any(a in temps for x in without for a, _, _ in x)  # TEMP epochs did travel before
+    src = p.source(mode)
+    assert "push down" in src and "push up" in src and "sf_xs_wait" in src and "sf_xs_signal" in src
+    assert "push down" not in q.source(mode)
+    p.compile(mode)

@@ -396,13 +396,13 @@ def run_ours(args):
         dist.destroy_process_group()
 
 
-def oracle_step_time(prog, nz_s, seed=4):
+def oracle_step_time(prog, nz_s, seed=4, parallel=False):
     from oracle import OracleProgram, dense_arrays
     from synth.programs import resize
     g = prog["grid"]
     sub = resize(prog, g["nx"], g["ny"], nz_s)
     arrs = dense_arrays(sub, seed)
-    o = OracleProgram(sub)
+    o = OracleProgram(sub, parallel=parallel)
     t0 = time.perf_counter()
     o.run(arrs)
     return time.perf_counter() - t0, sub
@@ -422,9 +422,20 @@ def cpu_baseline(args, budget_s=15.0, steps=1):
         ts.append(t)
     t = sum(ts) / len(ts)
     upd = g["nx"] * g["ny"] * nz_s * len(prog["kernels"])
-    return {"value": upd / t, "unit": UNIT, "cores": 1, "kind": "oracle",
-            "sample": f"{args.workload} program on a {g['nx']}x{g['ny']}x{nz_s} z-(sub)slab, mean of {steps} "
-                      f"step(s), serial C oracle (-O2 -ffp-contract=off), {t:.2f} s per step"}
+    out = {"value": upd / t, "unit": UNIT, "cores": 1, "kind": "oracle",
+           "sample": f"{args.workload} program on a {g['nx']}x{g['ny']}x{nz_s} z-(sub)slab, mean of {steps} "
+                     f"step(s), serial C oracle (-O2 -ffp-contract=off), {t:.2f} s per step"}
+    # context only: the OpenMP build of the same loop nest on every
+    # host core, on the whole per-GPU slab (identical results, tests/test_oracle_pins.py)
+    try:
+        cores = os.cpu_count() or 1
+        tp, _ = oracle_step_time(prog, g["nz"], parallel=True)
+        out["parallel"] = {"value": g["nx"] * g["ny"] * g["nz"] * len(prog["kernels"]) / tp,
+                           "unit": UNIT, "cores": cores,
+                           "kind": "oracle loop nest, OpenMP over z (-fopenmp), one step"}
+    except Exception as e:  # reported, not fatal
+        out["parallel"] = f"unavailable: {e}"
+    return out
 
 
 def run_reference(args):

@@ -66,6 +66,16 @@ static void clip_box(const or_grid *g, const long *box, long r[6]) {
     }
 }
 
+/* Built with -fopenmp (liboracle_omp.so, the parallel CPU baseline of SURVEY.md
+ * §8(d)) the planes of one statement are split across threads; every point is
+ * still evaluated by the same expression in the same order (points of one
+ * statement are independent, reading R3), so the result is identical. */
+#ifdef _OPENMP
+#define OR_PARALLEL_FOR _Pragma("omp parallel for schedule(static)")
+#else
+#define OR_PARALLEL_FOR
+#endif
+
 /* One generic body per storage type; REAL is the arithmetic type.
  * T(term) = coef * a[p+oa]  or  (coef * a[p+oa]) * b[p+ob]            (R4) */
 #define OR_DEFINE(NAME, STORE, REAL)                                                   \
@@ -85,6 +95,7 @@ static void clip_box(const or_grid *g, const long *box, long r[6]) {
                     if (S->box[2 * d] > q[2 * d]) q[2 * d] = S->box[2 * d];            \
                     if (S->box[2 * d + 1] < q[2 * d + 1]) q[2 * d + 1] = S->box[2 * d + 1]; \
                 }                                                                      \
+            OR_PARALLEL_FOR                                                            \
             for (long k = q[4]; k < q[5]; ++k)                                         \
                 for (long j = q[2]; j < q[3]; ++j)                                     \
                     for (long i = q[0]; i < q[1]; ++i) {                               \

@@ -21,7 +21,9 @@ import numpy as np
 
 _HERE = os.path.dirname(os.path.abspath(__file__))
 _LIB_PATH = os.path.join(_HERE, "liboracle.so")
+_LIB_OMP_PATH = os.path.join(_HERE, "liboracle_omp.so")  # same source, -fopenmp
 _lib = None
+_lib_omp = None
 
 
 class OrTap(ctypes.Structure):
@@ -45,21 +47,23 @@ class OrGrid(ctypes.Structure):
 
 
 def build_oracle(force: bool = False) -> str:
-    """Compile oracle.c with the flags reading R4 requires (no FMA contraction)."""
+    """Compile oracle.c with the flags reading R4 requires (no FMA contraction); also
+    the OpenMP build of the same source (parallel CPU baseline)."""
     src = os.path.join(_HERE, "oracle.c")
-    if force or not os.path.exists(_LIB_PATH) or \
-            os.path.getmtime(_LIB_PATH) < max(os.path.getmtime(src),
-                                               os.path.getmtime(os.path.join(_HERE, "oracle.h"))):
-        subprocess.check_call(["gcc", "-O2", "-ffp-contract=off", "-fno-fast-math", "-std=c11",
-                               "-fPIC", "-shared", "-o", _LIB_PATH, src])
+    for path, extra in ((_LIB_PATH, []), (_LIB_OMP_PATH, ["-fopenmp"])):
+        if force or not os.path.exists(path) or \
+                os.path.getmtime(path) < max(os.path.getmtime(src),
+                                             os.path.getmtime(os.path.join(_HERE, "oracle.h"))):
+            subprocess.check_call(["gcc", "-O2", "-ffp-contract=off", "-fno-fast-math", "-std=c11",
+                                   "-fPIC", "-shared"] + extra + ["-o", path, src])
     return _LIB_PATH
 
 
-def load_library():
-    global _lib
-    if _lib is None:
+def load_library(parallel: bool = False):
+    global _lib, _lib_omp
+    if (_lib_omp if parallel else _lib) is None:
         build_oracle()
-        lib = ctypes.CDLL(_LIB_PATH)
+        lib = ctypes.CDLL(_LIB_OMP_PATH if parallel else _LIB_PATH)
         for name, real in (("f64", ctypes.c_double), ("f32", ctypes.c_float)):
             f = getattr(lib, f"oracle_run_{name}")
             f.argtypes = [ctypes.POINTER(OrGrid), ctypes.c_int, ctypes.POINTER(ctypes.POINTER(real)),
@@ -74,14 +78,18 @@ def load_library():
             ctypes.POINTER(OrGrid), ctypes.c_int, ctypes.POINTER(ctypes.POINTER(ctypes.c_float)),
             ctypes.c_int, ctypes.POINTER(OrStmt)]
         lib.oracle_run_f32_in_f64.restype = ctypes.c_int
-        _lib = lib
-    return _lib
+        if parallel:
+            _lib_omp = lib
+        else:
+            _lib = lib
+    return _lib_omp if parallel else _lib
 
 
 class OracleProgram:
     """The original program, flattened to statements in program order."""
 
-    def __init__(self, prog: dict):
+    def __init__(self, prog: dict, parallel: bool = False):
+        self.parallel = parallel  # OpenMP build over z (identical results, reading R3)
         self.prog = prog
         self.dtype = prog["dtype"]
         g = prog["grid"]
@@ -166,7 +174,7 @@ class OracleProgram:
         n: interior size of the arrays if they are a window, not the program grid;
         origin: global coordinates of the window's interior point (0,0,0).
         """
-        lib = load_library()
+        lib = load_library(self.parallel)
         self._set_origin(origin)
         grid = self._grid(n)
         real = ctypes.c_double if self.dtype == "f64" else ctypes.c_float

@@ -455,3 +455,17 @@ def test_window_evaluation_matches_full_grid(cfg):
                             slice(h[1] + lo[1] - o[1], h[1] + hi[1] - o[1]),
                             slice(h[0] + lo[0] - o[0], h[0] + hi[0] - o[0]))
             assert np.array_equal(win[nm][sl(origin)], full[nm][sl((0, 0, 0))]), (cfg, origin, nm)
+
+
+@pytest.mark.parametrize("cfg", ["C2", "C3", "C5"])
+def test_openmp_build_identical(cfg):
+    """The OpenMP build of the oracle (parallel CPU baseline) splits the
+    planes of one statement across threads; results are bit-identical to the serial one."""
+    prog = {"C2": lambda: P.c2(nx=24, ny=20, nz=18), "C3": lambda: P.c3(nx=24, ny=20, nz=18),
+            "C5": lambda: P.c5(nx=24, ny=20, nz=18)}[cfg]()
+    a = dense_arrays(prog, 6)
+    b = {k: v.copy() for k, v in a.items()}
+    OracleProgram(prog).run(a)
+    OracleProgram(prog, parallel=True).run(b)
+    for k in a:
+        assert a[k].tobytes() == b[k].tobytes(), k

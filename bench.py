@@ -46,7 +46,7 @@ def load_workload(name):
         if os.path.exists(plan_path):
             pj = json.load(open(plan_path))
             prog["plans"]["fused"] = pj["groups"]
-            prog["plan_configs"] = {"fused": pj.get("configs")}
+            prog["plan_configs"] = {"fused": pj.get("configs"), "unfused": pj.get("unfused_configs")}
         return prog
     prog = P.CONFIGS[name]()
     path = os.path.join(ROOT, "configs", f"{name.lower()}_plan.json")
@@ -69,6 +69,10 @@ def apply_tuning(p, prog, plan="fused"):
         for i, c in enumerate(cfgs):
             if c:
                 p.tune("fused", i, c)
+    # the unfused baseline's per-kernel configurations, when tuned
+    for i, c in enumerate(tuned_configs(prog, "unfused") or []):
+        if c:
+            p.tune("unfused", i, c)
 
 
 def plan_of(prog, name="fused"):

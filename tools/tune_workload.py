@@ -29,6 +29,7 @@ def main():
     ap.add_argument("plans", nargs="+")
     ap.add_argument("--out", required=True)
     ap.add_argument("--iters", type=int, default=5)
+    ap.add_argument("--quick", action="store_true", help="reduced candidate set (unfused kernels)")
     a = ap.parse_args()
     prog = bench.load_workload(a.workload)
     dev = torch.device("cuda:0")
@@ -38,8 +39,11 @@ def main():
            "plans": {}}
     t0 = time.time()
     for name in a.plans:
+        # plan name "unfused": the original kernels, one launch each (the baseline)
+        mode = "unfused" if name == "unfused" else "fused"
         p = Program(prog)
-        p.set_plan(prog["plans"][name])
+        if mode == "fused":
+            p.set_plan(prog["plans"][name])
         if tensors is None:
             p.allocate(dev, fill=0.0)
             bench.fill_inputs(p, prog, dev, 0, prog["grid"]["ghost"][2])
@@ -49,14 +53,14 @@ def main():
                 p.bind(n, t)
 
         def timeit(i):
-            p.run_launch("fused", i)
+            p.run_launch(mode, i)
             torch.cuda.synchronize()
             ts = []
             for _ in range(a.iters):
                 flush.sum()
                 s, e = torch.cuda.Event(True), torch.cuda.Event(True)
                 s.record()
-                p.run_launch("fused", i)
+                p.run_launch(mode, i)
                 e.record()
                 torch.cuda.synchronize()
                 ts.append(s.elapsed_time(e) * 1e3)
@@ -64,8 +68,8 @@ def main():
 
         cfgs, us = [], []
         memo = {}
-        for i in range(p.n_launches("fused")):
-            r = p.report("fused", i)
+        for i in range(p.n_launches(mode)):
+            r = p.report(mode, i)
             if r["grid_ctas"] == 0:
                 cfgs.append(None)
                 us.append(0.0)
@@ -75,23 +79,30 @@ def main():
                    r["flops_alg"], r["z_below"], r["z_above"])
             if sig in memo:
                 best_c = memo[sig]
-                p.tune("fused", i, best_c)
+                if best_c:
+                    p.tune(mode, i, best_c)
                 best_t = timeit(i)
             else:
                 best_t, best_c = timeit(i), None
                 chooser_t = best_t
-                for c in candidates(prog["grid"]["ny"]):
+                cands = candidates(prog["grid"]["ny"])
+                if a.quick:
+                    cands = [c for c in cands if c["block_cby"] == 1 and c["block_x"] * c["block_y"] in (2, 4)
+                             and c["prefetch"] == 2]
+                for c in cands:
                     c = dict(c)
-                    for zc in (16, 32):
+                    for zc, pf in ((16, 2), (32, 1)) if a.quick else ((16, None), (32, None)):
                         c["zchunk"] = zc
+                        if pf:
+                            c["prefetch"] = pf
                         try:
-                            p.tune("fused", i, c)
+                            p.tune(mode, i, c)
                             t = timeit(i)
                         except StencilError:
                             continue
                         if t < best_t:
                             best_t, best_c = t, dict(c)
-                p.tune("fused", i, best_c)
+                p.tune(mode, i, best_c)
                 memo[sig] = best_c
                 print(f"{name} group {i}: chooser {chooser_t:.1f} us -> {best_t:.1f} us {best_c} "
                       f"({time.time() - t0:.0f} s)", flush=True)

@@ -116,12 +116,24 @@ def test_zqueue_bitexact(cuda_device, zqueue):
 
 
 def test_c2_full_size(cuda_device):
-    """BASELINE configs[1] at its full size (256^3 fp64), perf build, vs the oracle."""
+    """BASELINE configs[1] at its full size (256^3 fp64), perf build, vs the oracle: the
+    model-chosen tiles, then the bench's tuned per-launch configurations (fused and the
+    tuned unfused baseline)."""
+    import sys
+    sys.path.insert(0, os.path.dirname(os.path.dirname(os.path.abspath(__file__))))
+    import bench
+    from _harness import gpu_program
     prog = P.c2()
     ref = oracle_outputs(prog, seed=2)
     for mode in ("unfused", "fused"):
         got = gpu_run(prog, mode, 2, plan=prog["plans"]["fused"])
         assert_close(prog, got, ref)
+    bprog = bench.load_workload("C2")
+    for mode in ("unfused", "fused"):
+        p = gpu_program(bprog, plan=bprog["plans"]["fused"])
+        bench.apply_tuning(p, bprog)
+        got = gpu_run(bprog, mode, 2, program=p)
+        assert_close(bprog, got, ref)
 
 
 def _c4_small():
@@ -133,10 +145,12 @@ def _c4_small():
     return prog
 
 
-def test_c4_full_size_bench_configuration(cuda_device):
+@pytest.mark.parametrize("mode", ["fused", "unfused"])
+def test_c4_full_size_bench_configuration(cuda_device, mode):
     """BASELINE configs[3] at its full size (1280x32x256 fp64) in exactly the launch
-    configuration bench.py times (frozen plan + tuned tiles, perf build), against the
-    full serial oracle (~5 s on the host)."""
+    configuration bench.py times (frozen plan + tuned tiles, perf build; for "unfused"
+    the tuned per-kernel configurations of the baseline the speedup is quoted against),
+    against the full serial oracle (~5 s on the host)."""
     import sys
     sys.path.insert(0, os.path.dirname(os.path.dirname(os.path.abspath(__file__))))
     import bench
@@ -145,7 +159,7 @@ def test_c4_full_size_bench_configuration(cuda_device):
     ref = oracle_outputs(prog, seed=3)
     p = gpu_program(prog, plan=prog["plans"]["fused"])
     bench.apply_tuning(p, prog)
-    got = gpu_run(prog, "fused", 3, program=p)
+    got = gpu_run(prog, mode, 3, program=p)
     assert_close(prog, got, ref)
 
 
@@ -200,7 +214,8 @@ def test_zwave_full_size_c4(cuda_device):
 
 
 @pytest.mark.parametrize("workload,plan,w", [("C5", "fused", 24), ("C3", "measured", 32),
-                                             ("C3", "fission_fused", 32)])
+                                             ("C3", "fission_fused", 32), ("C5", "unfused", 24),
+                                             ("C3", "unfused", 32)])
 def test_full_size_sampled_bench_configuration(cuda_device, workload, plan, w):
     """BASELINE configs[2] (C3, 512^3 fp32) and configs[4]'s per-GPU grid (C5, 1024x1024x128
     fp64) at full size, in the launch configuration bench.py times (plan + tuned tiles,
@@ -220,12 +235,13 @@ def test_full_size_sampled_bench_configuration(cuda_device, workload, plan, w):
     N = (g["nx"], g["ny"], g["nz"])
     h = tuple(g["ghost"])
     m = accumulated_reach(prog)
-    p = gpu_program(prog, plan=bench.plan_of(prog, plan))
-    bench.apply_tuning(p, prog, plan)
+    unfused = plan == "unfused"  # the tuned unfused baseline (its configurations only)
+    p = gpu_program(prog, plan=bench.plan_of(prog, "fused" if unfused else plan))
+    bench.apply_tuning(p, prog, "fused" if unfused else plan)
     dev = torch.device("cuda:0")
     p.allocate(dev, fill=0.0)
     bench.fill_inputs(p, prog, dev, 0, h[2])
-    p.run_fused()
+    p.run_unfused() if unfused else p.run_fused()
     torch.cuda.synchronize()
     outs = [a["name"] for a in prog["arrays"] if a["role"] in ("out", "inout")]
     orc = OracleProgram(prog)

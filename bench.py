@@ -188,6 +188,12 @@ def run_ours(args):
     fill_inputs(p, prog, dev, rank * nz, zhalo)
     if xpush:
         p.connect_peers(rank, world)
+        # every rank's modules are loaded before any kernel can wait on a neighbour
+        # (a neighbour still compiling would otherwise look like a dead rank)
+        p.load("fused")
+        p.load("unfused")
+        torch.cuda.synchronize(dev)
+        dist.barrier()
     stream = torch.cuda.current_stream(dev)
     n_pts = prog["grid"]["nx"] * prog["grid"]["ny"] * nz  # per GPU
     n_kernels = len(prog["kernels"])
@@ -229,6 +235,24 @@ def run_ours(args):
     step_ms = s.elapsed_time(e) / args.steps
     clocks = sampler.stop()
     step_ms = max_over_ranks(step_ms)
+    # sustained: >= 1 s of back-to-back steps (at least 200), one CUDA event per step
+    # boundary on the launching stream; median / mean per step beside the K-step headline
+    sus_n = max(200, int(1.0 / max(step_ms * 1e-3, 1e-6)) + 1)
+    sus_ev = [torch.cuda.Event(enable_timing=True) for _ in range(sus_n + 1)]
+    sus_sampler = ClockSampler(dev.index)
+    sus_sampler.start()
+    time.sleep(0.25)
+    barrier()
+    sus_ev[0].record(stream)
+    for k in range(sus_n):
+        p.run_fused(stream)
+        sus_ev[k + 1].record(stream)
+    barrier()
+    sus_clocks = sus_sampler.stop()
+    per_step = [sus_ev[k].elapsed_time(sus_ev[k + 1]) for k in range(sus_n)]
+    sustained = {"steps": sus_n, "ms_per_step_median": max_over_ranks(statistics.median(per_step)),
+                 "ms_per_step_mean": max_over_ranks(sus_ev[0].elapsed_time(sus_ev[-1]) / sus_n),
+                 "timed_s": sus_ev[0].elapsed_time(sus_ev[-1]) * 1e-3, "clocks": sus_clocks}
     # the same step captured once as a CUDA graph and replayed K times (SURVEY.md §8(d)
     # timing protocol; S7): launch overhead off the host, same kernels
     graph_ms = None
@@ -384,11 +408,14 @@ def run_ours(args):
                                  "predicted_traffic_reduction": 1 - alg_step / alg_step_u},
             "e2e": {"value": updates / (e2e_ms * 1e-3), "unit": UNIT, "h2d_bytes_per_step": h2d,
                     "d2h_bytes_per_step": d2h, "ms_per_step": e2e_ms},
-            # N > 1: a launch that receives ghost planes runs as interior + 2 boundary launches
+            "sustained": dict(sustained, value=updates / (sustained["ms_per_step_median"] * 1e-3),
+                              frac_of_peak=alg_step / (sustained["ms_per_step_median"] * 1e-3) / 1e9 / peak,
+                              note="median of per-step CUDA events over >= 1 s of back-to-back steps"),
             "graph_replay": {"ms_per_step": graph_ms, "note": "one fused step captured as a CUDA "
                              "graph, replayed K times (same kernels; not the headline)"},
-            "gpu_launches": args.steps * sum(3 if world > 1 and p.exchange_plan("fused", i) else 1
-                                             for i in live_f),
+            # this library's kernels in the timed region (sp_run_launch_count: on N > 1 a
+            # launch that receives ghost planes is an interior + one boundary launch)
+            "gpu_launches": args.steps * p.launch_count("fused"),
             "clocks": clocks,
             "wall_s_timed": wall,
         }
@@ -471,6 +498,39 @@ def run_reference(args):
     }), flush=True)
 
 
+def _free_port():
+    import socket
+    sk = socket.socket()
+    sk.bind(("127.0.0.1", 0))
+    port = sk.getsockname()[1]
+    sk.close()
+    return port
+
+
+def ensure_world(args):
+    """One process per GPU.  Under torchrun (WORLD_SIZE set) the world must equal --gpus;
+    without it, --gpus N > 1 re-executes this script under torch.distributed.run with N
+    ranks on this node (the driver's own launch line) and exits with its status, so a
+    multi-GPU request never silently benchmarks one GPU."""
+    env = os.environ.get("WORLD_SIZE")
+    if env is not None:
+        if int(env) != args.gpus:
+            sys.exit(f"bench.py: --gpus {args.gpus} but WORLD_SIZE={env}: refusing to report a "
+                     f"{env}-rank run as {args.gpus} GPUs")
+        return
+    if args.gpus <= 1:
+        return
+    if args.impl == "ours":
+        import torch
+        have = torch.cuda.device_count()
+        if have < args.gpus:
+            sys.exit(f"bench.py: --gpus {args.gpus} requested but only {have} CUDA device(s) visible")
+    cmd = [sys.executable, "-m", "torch.distributed.run", "--nnodes=1",
+           f"--nproc-per-node={args.gpus}", "--master-addr=127.0.0.1",
+           f"--master-port={_free_port()}", os.path.abspath(__file__)] + sys.argv[1:]
+    sys.exit(subprocess.call(cmd))
+
+
 def main():
     ap = argparse.ArgumentParser()
     ap.add_argument("--gpus", type=int, default=1)
@@ -486,6 +546,9 @@ def main():
     args = ap.parse_args()
     if args.warmup < 3:
         args.warmup = 3
+    if args.gpus < 1:
+        sys.exit("bench.py: --gpus must be >= 1")
+    ensure_world(args)
     if args.impl == "reference":
         run_reference(args)
     else:

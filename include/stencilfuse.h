@@ -346,6 +346,13 @@ sp_status run_unfused(stencil_program *prog, sp_stream stream);
 sp_status run_fused(stencil_program *prog, sp_stream stream);
 /* One launch of a mode (profiling / per-kernel timing); no exchange. */
 sp_status sp_run_launch(stencil_program *prog, int32_t mode, int32_t launch, sp_stream stream);
+/* Number of kernel launches one run_unfused (mode 0) / run_fused (mode 1) call
+ * issues with the current communicator and options: one per live launch; on
+ * several ranks a launch that receives ghost planes first (sp_plan_exchange) is
+ * an interior launch plus one boundary launch covering both slab ends (one
+ * launch when its interior is empty); under "zwave" one per non-empty wave of
+ * each launch.  NCCL's own kernels are not counted.  Host-only. */
+sp_status sp_run_launch_count(stencil_program *prog, int32_t mode, int32_t *n);
 
 /* Exchange `depth` ghost planes of each listed array with the z-neighbours
  * (ncclSend/ncclRecv grouped; planes are contiguous, no packing).  Requires

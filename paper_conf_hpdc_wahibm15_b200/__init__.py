@@ -397,6 +397,12 @@ class Program:
     def run_launch(self, mode, i, stream=None):
         _check(lib().sp_run_launch(self.handle, self._mode(mode), i, _stream_handle(stream)))
 
+    def launch_count(self, mode):
+        """Kernel launches one run_unfused / run_fused call issues (sp_run_launch_count)."""
+        n = ctypes.c_int32()
+        _check(lib().sp_run_launch_count(self.handle, self._mode(mode), ctypes.byref(n)))
+        return n.value
+
     def exchange_halos(self, names, depth, stream=None):
         arr = (ctypes.c_int32 * len(names))(*[self.index[n] for n in names])
         _check(lib().exchange_halos(self.handle, len(names), arr, depth, _stream_handle(stream)))

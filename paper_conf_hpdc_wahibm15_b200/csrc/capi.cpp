@@ -183,6 +183,45 @@ static void run_waves(stencil_program *p, Mode &m, void *stream) {
     }
 }
 
+// kernel launches one run_* call issues under the current communicator and options
+// (mirrors run_mode / run_waves: a launch that receives ghost planes on several
+// ranks is an interior launch plus one two-range boundary launch, or one launch
+// when its interior is empty)
+static int count_launches(stencil_program *p, int mode) {
+    Mode &m = mode_of(p, mode);
+    const bool multi = p->comm && p->comm->nranks > 1;
+    const int nz = (int)p->grid.nz_local;
+    int n = 0;
+    if (mode == 1 && p->opt.zwave > 0 && !multi) {
+        if (m.wave_off.size() != m.launches.size()) wave_offsets(p, m);
+        const int S = p->opt.zwave;
+        int maxoff = 0;
+        for (int o : m.wave_off) maxoff = std::max(maxoff, o);
+        const int nw = (nz + maxoff + S - 1) / S;
+        for (int w = 0; w < nw; ++w)
+            for (size_t i = 0; i < m.launches.size(); ++i) {
+                if (m.launches[i].dead) continue;
+                const int z0 = std::max(0, w * S - m.wave_off[i]);
+                const int z1 = std::min(nz, (w + 1) * S - m.wave_off[i]);
+                n += z1 > z0;
+            }
+        return n;
+    }
+    if (multi && !m.xsched_ok) exchange_schedule(p, m);
+    for (size_t i = 0; i < m.launches.size(); ++i) {
+        const Launch &L = m.launches[i];
+        if (L.dead || L.zc <= 0) continue;
+        if (!multi || m.xsched[i].empty()) {
+            n += 1;
+            continue;
+        }
+        int zb, ze;
+        interior_planes(p, L, m.xsched[i], &zb, &ze);
+        n += ze > zb ? 2 : 1;
+    }
+    return n;
+}
+
 static void run_mode(stencil_program *p, int mode, void *stream) {
     Mode &m = mode_of(p, mode);
     load_mode(p, m);
@@ -379,6 +418,7 @@ sp_status sp_program_set_option(stencil_program *p, const char *key, int64_t v) 
         else if (k == "zwave") o.zwave = (int)v;
         else if (k == "zwave_streams") o.zwave_streams = std::max(1, std::min(8, (int)v));
         else if (k == "xpush") o.xpush = v != 0;
+        else if (k == "fastpath") o.fastpath = v != 0;
         else if (k == "regcap") o.regcap = (int)std::min<int64_t>(v, 2);
         else if (k == "l2_flush") {}
         else fail(SP_E_ARG, "unknown option '" + k + "'");
@@ -592,6 +632,13 @@ sp_status sp_run_launch(stencil_program *p, int32_t mode, int32_t i, sp_stream s
         load_mode(p, m);
         if (p->comm && p->comm->nranks > 1) p->no_pdl = true;
         launch(p, m, i, stream);
+    });
+}
+
+sp_status sp_run_launch_count(stencil_program *p, int32_t mode, int32_t *n) {
+    return guard([&] {
+        if (!p || !n) fail(SP_E_ARG, "null argument");
+        *n = count_launches(p, mode);
     });
 }
 

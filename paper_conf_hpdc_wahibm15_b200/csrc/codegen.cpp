@@ -31,6 +31,7 @@
 #include <cstdio>
 #include <cstdlib>
 #include <cstring>
+#include <climits>
 #include <functional>
 #include <set>
 #include <sstream>
@@ -570,6 +571,34 @@ std::string generate_launch(const stencil_program *p, Launch &L, int index, bool
         o << "      }\n    }\n";
     }
 
+    // Step body, emitted twice when possible: FP (fast step) = an interior tile at a
+    // step where every statement's plane lies inside the slab's global interior (and,
+    // for stored statements, inside the chunk): every range / ghost / store predicate
+    // is then the constant true and the compiler drops those branches; the general
+    // body serves edge tiles, warm-up steps and the chunk's last planes.  Both bodies
+    // evaluate the same expressions in the same order (bit-identical results).
+    bool any_boxed = false;
+    for (const Stage &G : L.st)
+        if (G.needed && p->stmts[G.gid].boxed) any_boxed = true;
+    const bool spec = p->opt.fastpath && !any_boxed;
+    if (spec) {
+        int smin = INT32_MAX, kst0 = INT32_MIN;
+        int lmin = INT32_MAX, lmax = INT32_MIN, slmin = INT32_MAX, slmax = INT32_MIN;
+        for (const Stage &G : L.st) {
+            if (!G.needed) continue;
+            kst0 = std::max(kst0, G.loff - G.lead);
+            lmin = std::min(lmin, G.lead);
+            lmax = std::max(lmax, G.lead);
+            if (G.stored) { slmin = std::min(slmin, G.lead); slmax = std::max(slmax, G.lead); }
+        }
+        (void)smin;
+        o << "    // fast-step window [sf_k0, sf_k1) of this chunk (see codegen.cpp)\n";
+        o << "    int sf_k0 = max(" << kst0 << ", ZLO - Z0 - (" << lmin << ")), sf_k1 = min(zc, ZHI - Z0 - ("
+          << lmax << "));\n";
+        if (slmin != INT32_MAX)
+            o << "    sf_k0 = max(sf_k0, -(" << slmin << ")); sf_k1 = min(sf_k1, zc - (" << slmax << "));\n";
+    }
+    auto emit_body = [&](const bool FP) {
     std::set<int> dirty;
     for (size_t mi = 0; mi < L.st.size(); ++mi) {
         const int m = (int)mi;
@@ -639,21 +668,26 @@ std::string generate_launch(const stencil_program *p, Launch &L, int index, bool
             o << "        }\n      }\n";
         }
         o << "      const int q = k + (" << G.lead << ");\n";
-        o << "      if (q >= (" << G.loff << ") && q <= zc - 1 + (" << G.lead << ")) {\n";
+        if (FP) o << "      {\n";
+        else o << "      if (q >= (" << G.loff << ") && q <= zc - 1 + (" << G.lead << ")) {\n";
         o << "        const int gz = Z0 + q;\n";
         const bool boxed = p->stmts[G.gid].boxed;
         // in-box tests of this statement (the whole interior unless boxed)
         const std::string BX0 = boxed ? num(sbox(G, 0)) : "0", BX1 = boxed ? num(sbox(G, 1)) : "NX";
         const std::string BY0 = boxed ? num(sbox(G, 2)) : "0", BY1 = boxed ? num(sbox(G, 3)) : "NY";
-        if (boxed)
+        if (FP)
+            o << "        const bool zin = true;  // fast step\n";
+        else if (boxed)
             o << "        const bool zin = gz >= (" << sbox(G, 4) << ") && gz < (" << sbox(G, 5)
               << ");  // loop bounds (R2')\n";
         else
             o << "        const bool zin = gz >= ZLO && gz < ZHI;\n";
-        o << "        const bool zal = gz + OZA >= 0 && gz + OZA < ZA;\n";
+        o << "        const bool zal = " << (FP ? "true" : "gz + OZA >= 0 && gz + OZA < ZA") << ";\n";
         o << "        T *const gpl = p.arr[" << L.arr_slot[G.out] << "] + (long long)(gz + OZA) * PLANE;\n";
-        if (G.stored) o << "        const bool zst = q >= 0 && q < zc;\n";
-        if (boxed)
+        if (G.stored) o << "        const bool zst = " << (FP ? "true" : "q >= 0 && q < zc") << ";\n";
+        if (FP)
+            o << "        const bool fast = true;\n";
+        else if (boxed)
             o << "        const bool fast = X0 >= " << BX0 << " && X0 + TX <= " << BX1 << " && Y0 >= "
               << BY0 << " && Y0 + TY <= " << BY1 << " && zin;\n";
         else
@@ -909,6 +943,16 @@ std::string generate_launch(const stencil_program *p, Launch &L, int index, bool
         }
         o << "      }\n    }\n";
         if (G.keep == Keep::Smem) dirty.insert(m);
+    }
+    };
+    if (spec) {
+        o << "    if (tile_in && k >= sf_k0 && k < sf_k1) {\n";
+        emit_body(true);
+        o << "    } else {\n";
+        emit_body(false);
+        o << "    }\n";
+    } else {
+        emit_body(false);
     }
     if (tma) {
         o << "    __syncwarp();\n";

@@ -119,14 +119,18 @@ void exchange_schedule(const stencil_program *p, Mode &m) {
     for (size_t i = 0; i < n; ++i) {
         const Launch &L = m.launches[i];
         if (L.dead) continue;
-        for (const Input &I : L.in) {
-            const int b = std::max(0, -I.qlo), u = std::max(0, I.ahi);
-            if (!b && !u) continue;
-            if (first[I.arr] < 0) first[I.arr] = writer[I.arr] >= 0 ? (int)i : first_live;
-            below[I.arr] = std::max(below[I.arr], b);
-            above[I.arr] = std::max(above[I.arr], u);
-            readers[I.arr].push_back((int)i);
-        }
+        auto read = [&](int arr, int b, int u) {
+            if (!b && !u) return;
+            if (first[arr] < 0) first[arr] = writer[arr] >= 0 ? (int)i : first_live;
+            below[arr] = std::max(below[arr], b);
+            above[arr] = std::max(above[arr], u);
+            readers[arr].push_back((int)i);
+        };
+        for (const Input &I : L.in) read(I.arr, std::max(0, -I.qlo), std::max(0, I.ahi));
+        // R2': a boxed statement evaluated on planes beyond the slab (z warm-up below,
+        // lead above) loads its array's previous value there outside its box
+        for (const Stage &G : L.st)
+            if (G.needed && p->stmts[G.gid].boxed) read(G.out, std::max(0, -G.loff), std::max(0, G.lead));
         for (const Stage &G : L.st)
             if (G.stored) {
                 flush(G.out);

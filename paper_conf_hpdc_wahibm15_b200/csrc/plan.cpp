@@ -514,6 +514,12 @@ static void live_out(const stencil_program *p, bool fused,
                     if (lastw[a].first >= 0 && lastw[a].first < (int)g)
                         stored[lastw[a].first].insert(lastw[a].second);
                 }
+            // R2': a statement with loop bounds overwrites only its box; every other
+            // point keeps the previous value, which it loads from memory (codegen) —
+            // so a boxed write reads the array like a tap does
+            if (S.boxed && !written_here.count(S.out) && lastw[S.out].first >= 0 &&
+                lastw[S.out].first < (int)g)
+                stored[lastw[S.out].first].insert(lastw[S.out].second);
             written_here.insert(S.out);
         }
         std::map<int, int> last;

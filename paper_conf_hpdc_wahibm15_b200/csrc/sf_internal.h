@@ -46,6 +46,7 @@ struct Options {
     int zwave = 0;          // z-wave schedule: planes per wave (0 = one launch per group per step)
     int zwave_streams = 2;  // waves in flight (streams) of the z-wave schedule
     int xpush = 0;  // several ranks: stores push in-step halo planes into the neighbours' ghosts
+    int fastpath = 1;  // emit a predicate-free step body for interior tiles / planes
     int regcap = 1; // recompile a few registers tighter when that adds a resident CTA:
                     // 0 never, 1 peer-push kernels, 2 every kernel
 };

@@ -73,3 +73,53 @@ def random_plans(rng, prog, count=3):
                 prev = c
         plans.append(groups)
     return plans
+
+
+def _fuses_boxed(prog, plan):
+    """Does some group hold a statement of a boxed kernel together with another statement?"""
+    boxed = {k["name"] for k in prog["kernels"] if k.get("box") is not None}
+    return any(len(g) > 1 and any(r.split(":")[0] in boxed for r in g) for g in plan)
+
+
+def legal_plans(rng, prog, want=4, tries=60):
+    """Up to `want` fusion plans the library accepts (host-side fusion_plan_set: partition,
+    order, R11/R2' hazards, resources), each with at least one multi-statement group:
+    the single group, the model's greedy plan, then random contiguous cuts.  Plans that
+    fuse a boxed kernel with another statement come first.  Returns (plans, rejected),
+    rejected = [(plan, sp_status)] for the candidates refused with a plan error."""
+    from paper_conf_hpdc_wahibm15_b200 import Program, StencilError
+    p = Program(prog)
+    cands = random_plans(rng, prog, count=tries)
+    try:
+        cands.insert(1, p.plan_greedy())
+    except StencilError:
+        pass
+    ok, rejected, seen = [], [], set()
+    for plan in cands:
+        key = tuple(tuple(g) for g in plan)
+        if key in seen or all(len(g) == 1 for g in plan):
+            continue
+        seen.add(key)
+        try:
+            p.set_plan(plan)
+        except StencilError as e:
+            rejected.append((plan, e.code))
+            continue
+        ok.append(plan)
+    ok.sort(key=lambda pl: not _fuses_boxed(prog, pl))  # stable: boxed fusions first
+    return ok[:want], rejected
+
+
+def fuzz_case(seed, boxes, max_draws=12):
+    """Seeded fuzz case: programs are drawn from one generator stream until one admits at
+    least two accepted fusion plans (boxed cases: the first of them fuses a boxed kernel
+    with another statement), so every case really runs fused plans.  Returns
+    (program, plans, rejected, draws)."""
+    rng = np.random.default_rng(100 * seed + boxes)
+    for draw in range(1, max_draws + 1):
+        prog = random_lib_program(rng, dtype="f32" if seed % 4 == 3 else "f64", boxes=boxes)
+        plans, rejected = legal_plans(rng, prog)
+        has_box = any(k.get("box") is not None for k in prog["kernels"])
+        if len(plans) >= 2 and (not boxes or (has_box and _fuses_boxed(prog, plans[0]))):
+            return prog, plans, rejected, draw
+    raise RuntimeError(f"fuzz seed {seed}: no program with fusable plans in {max_draws} draws")

@@ -369,3 +369,57 @@ def test_peer_push_ipc_processes(cuda_device, cfg, concurrent):
     for p in ps:
         p.join(timeout=60)
     assert all(v == "ok" for v in res.values()), res
+
+
+@pytest.mark.parametrize("ranks", [2, 3])
+def test_loopback_exchange_halos_rank_encoded(cuda_device, ranks):
+    """exchange_halos (§8(b)) unit test on in-process virtual ranks: every array's whole
+    allocated planes carry an exact code of (array, global plane, y, x); after
+    exchange_halos(depth) each rank's ghost planes equal its neighbours' interior
+    planes, and interior planes and true global ghost planes are untouched."""
+    import threading
+    import torch
+    from _nccl_worker import encoded
+    from paper_conf_hpdc_wahibm15_b200 import Comm, Program
+    nzl, depth = 7, 3
+    prog = P.c2(nx=40, ny=24, nz=nzl)
+    comms = Comm.loopback(ranks)
+    progs = []
+    for r in range(ranks):
+        p = Program(prog, comm=comms[r], nz_global=nzl * ranks, z_offset=r * nzl, zhalo=depth)
+        p.allocate(cuda_device)
+        oz = p.layout["origin_z"]
+        for aid, n in enumerate(p.names):
+            t = p.tensors[n]
+            for z in range(nzl):
+                t[oz + z].copy_(encoded(aid, r * nzl + z, t.shape[1:], t.device))
+        progs.append(p)
+    torch.cuda.synchronize()
+    errs = []
+
+    def drive(r):
+        try:
+            st = torch.cuda.Stream(device=cuda_device)
+            progs[r].exchange_halos(progs[r].names, depth, st)
+            st.synchronize()
+        except Exception as e:  # surfaced below
+            errs.append(e)
+
+    th = [threading.Thread(target=drive, args=(r,)) for r in range(ranks)]
+    for t in th:
+        t.start()
+    for t in th:
+        t.join()
+    assert not errs, errs
+    for r, p in enumerate(progs):
+        oz = p.layout["origin_z"]
+        for aid, n in enumerate(p.names):
+            t = p.tensors[n]
+            for z in range(-depth, nzl + depth):
+                gz = r * nzl + z
+                if 0 <= z < nzl:
+                    assert torch.equal(t[oz + z], encoded(aid, gz, t.shape[1:], t.device)), (r, n, z)
+                elif gz < 0 or gz >= nzl * ranks:
+                    assert torch.isnan(t[oz + z]).all(), (r, n, z)
+                else:
+                    assert torch.equal(t[oz + z], encoded(aid, gz, t.shape[1:], t.device)), (r, n, z)

@@ -2,6 +2,7 @@
 DDG/OEG edges, fission (Algorithm 2), plan legality, group analysis, the
 byte/flop model and NVRTC compilation of the generated sm_100a kernels."""
 import ctypes
+import os
 import re
 
 import pytest
@@ -9,6 +10,8 @@ import pytest
 from paper_conf_hpdc_wahibm15_b200 import Program, StencilError
 from paper_conf_hpdc_wahibm15_b200._abi import EXPORTS, LIB_PATH
 from synth import programs as P
+
+ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
 
 pytestmark = pytest.mark.host
 
@@ -507,3 +510,39 @@ def test_peer_push_schedule_and_codegen(mode):
     assert "push down" in src and "push up" in src and "sf_xs_wait" in src and "sf_xs_signal" in src
     assert "push down" not in q.source(mode)
     p.compile(mode)
+
+
+def test_fuzz_cases_run_fused_plans():
+    """Every GPU fuzz case (tests/test_gpu_fuzz.py) has >= 2 accepted fusion plans; boxed
+    cases fuse a boxed kernel with another statement (R2'); rejected candidates carry a
+    plan error (SP_E_PLAN_ORDER / _HAZARD / _RESOURCES)."""
+    from _fuzz import _fuses_boxed, fuzz_case
+    for boxes in (False, True):
+        for seed in range(12):
+            prog, plans, rejected, _ = fuzz_case(seed, boxes)
+            assert len(plans) >= 2
+            assert all(code in (4, 5, 6) for _, code in rejected)
+            assert all(any(len(g) > 1 for g in pl) for pl in plans)
+            if boxes:
+                assert _fuses_boxed(prog, plans[0])
+
+
+def test_run_launch_count():
+    """sp_run_launch_count: one launch per live launch on one rank; on several ranks the
+    launches that receive ghost planes split into interior + boundary (C4 fused, 2 ranks:
+    only the first launch receives the step-start exchange)."""
+    import json
+    from paper_conf_hpdc_wahibm15_b200 import Comm, Program
+    from synth.scale_les import c4
+    prog = c4(nx=64, ny=32, nz=32)
+    plan = json.load(open(os.path.join(ROOT, "configs", "c4_plan.json")))["groups"]
+    p = Program(prog)
+    p.set_plan(plan)
+    assert p.launch_count("fused") == len(plan)
+    assert p.launch_count("unfused") == len(prog["kernels"])
+    comms = Comm.loopback(2)
+    q = Program(prog, comm=comms[0], nz_global=64, z_offset=0, zhalo=4)
+    q.set_plan(plan)
+    recv = [i for i in range(len(plan)) if q.exchange_plan("fused", i)]
+    assert recv
+    assert q.launch_count("fused") == len(plan) + len(recv)

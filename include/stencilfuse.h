@@ -231,6 +231,9 @@ sp_status stencil_program_bind(stencil_program *prog, int32_t array, void *dev_p
  *               without spills): 0 never, 1 peer-push kernels (default), 2 all
  *   "l2pf"      TMA L2 prefetch of input planes this many steps beyond the
  *               shared-memory ring (default 1; 0 off)
+ *   "fastpath"  1: a second, predicate-free copy of the step body for interior
+ *               tiles/planes (fewer issued instructions, larger code); default 0
+ *   "minblocks" __launch_bounds__ minimum resident CTAs (ptxas register budget)
  *   "suspend_hint", "coef_const", "acc_split"   measured-off experiments
  *   "num_sms"   SM count assumed by the tile chooser (default 148)
  *   "l2_flush"  unused by the library (reserved) */
@@ -266,14 +269,54 @@ sp_status fusion_plan_set(stencil_program *prog, int32_t n_groups, const int32_t
  * With group_begin == NULL only *n_groups is returned.  Does not set the plan. */
 sp_status sp_plan_greedy(stencil_program *prog, int32_t cap, int32_t *n_groups,
                          int32_t *group_begin, sp_stmt_ref *members);
-/* GGA-lite plan search (the paper's grouping genetic
- * algorithm, whose encoding/operators are not in the paper): a
- * grouping GA over fission units (statements may be grouped out of program order
- * when independent), objective = the same launch-time model as sp_plan_greedy,
- * illegal groupings (cyclic group order, R11 hazards, no tile fitting shared
- * memory) rejected.  Seeded with the greedy plan, so its modelled cost is never
- * worse.  Deterministic for (generations, population, seed).  Output as in
- * sp_plan_greedy (call with group_begin == NULL first for *n_groups).  Host-only. */
+/* Lazy-fission plan search (the paper's search step,
+ * P:L140 §3.2.4 and §4.1).  Steps:
+ *   1. metadata pre-step: the objective is evaluated for every original kernel and
+ *      every fission piece (sp_fission_components) on its own ("lazy fission": the
+ *      pieces' metadata is gathered first);
+ *   2. exact DP over contiguous segmentations of the ORIGINAL kernels (no fission),
+ *      segments of at most max_group_kernels kernels — the live-out set (R6) of a
+ *      contiguous group depends on the group alone, so the DP optimum is exact;
+ *   3. a grouping GA over fission pieces whose kernels start unfissioned (a
+ *      kernel's pieces share one group until fission is applied to it): merge,
+ *      split, move, group-injection crossover and the lazy-fission operator, which
+ *      splits a kernel of a group that violates the shared-memory capacity;
+ *      seeded with the DP optimum, the unfused plan and sp_plan_greedy's plan.
+ *      Fitness is the paper's dynamic penalty
+ *          f_p(x) = f(x) + sum_i C_i delta_i - C_SM delta_SM
+ *      with f = sum of the groups' times (a violating group is charged its units'
+ *      pre-step times), delta_i = cyclic group order / in-group hazard (R11, R2') /
+ *      no tile fits (resources), C_SM = +c_sm when a kernel of the smem-violating
+ *      group can still be fissioned (the relaxation fission offers) and -c_sm when
+ *      not.  Independent statements may be grouped out of program order.
+ * Objective 0: this library's launch-time model (host only, deterministic for the
+ * options).  Objective 1: measured — every candidate group is JIT-compiled and timed
+ * on the current device with CUDA events on `stream` (median of `reps` launches,
+ * L2 flushed before each; the paper's empirical metadata, §3.2.1); the
+ * program's arrays must be bound, and their contents are overwritten.
+ * Output as sp_plan_greedy; `report` (nullable) receives costs and counts. */
+typedef struct {
+    int32_t generations;        /* GA generations (0: pre-step + DP + seeds only)            */
+    int32_t population;         /* GA population (clamped to >= 4)                            */
+    uint64_t seed;              /* GA random stream                                           */
+    int32_t objective;          /* 0 = launch-time model (host), 1 = measured on the device   */
+    int32_t max_group_kernels;  /* DP segment bound in original kernels (0 -> 8)              */
+    int32_t reps;               /* measured: timed launches per group, median (0 -> 5)        */
+    double c_violation;         /* C_i per violated constraint, x the unfused plan cost (0 -> 1) */
+    double c_sm;                /* |C_SM|, x the unfused plan cost (0 -> 0.5)                  */
+} sp_search_options;
+typedef struct {
+    double cost_us;             /* objective of the returned plan                             */
+    double dp_cost_us;          /* best contiguous unfissioned plan (step 2)                  */
+    double unfused_cost_us;     /* one group per original kernel                              */
+    int32_t groups_evaluated;   /* distinct groups the objective evaluated                    */
+    int32_t fissioned_kernels;  /* kernels whose pieces the returned plan separates           */
+    int32_t generations_run;
+} sp_search_report;
+sp_status sp_plan_search_ex(stencil_program *prog, const sp_search_options *opts, sp_stream stream,
+                            int32_t cap, int32_t *n_groups, int32_t *group_begin, sp_stmt_ref *members,
+                            sp_search_report *report);
+/* sp_plan_search_ex with the model objective and default constants.  Host-only. */
 sp_status sp_plan_search(stencil_program *prog, int32_t generations, int32_t population, uint64_t seed,
                          int32_t cap, int32_t *n_groups, int32_t *group_begin, sp_stmt_ref *members);
 

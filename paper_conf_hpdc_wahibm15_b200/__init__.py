@@ -15,7 +15,8 @@ import ctypes
 import os
 
 from ._abi import (SP_F32, SP_F64, ROLE, SpArrayDesc, SpEdge, SpGrid, SpGroupReport, SpKernel,
-                   SpLayout, SpStmt, SpStmtRef, SpTerm, SpTap, SpTileConfig, lib)
+                   SpLayout, SpSearchOptions, SpSearchReport, SpStmt, SpStmtRef, SpTerm, SpTap,
+                   SpTileConfig, lib)
 
 __all__ = ["Program", "Comm", "StencilError", "lib"]
 
@@ -319,6 +320,28 @@ class Program:
         names = [k["name"] for k in self.prog["kernels"]]
         return [[f"{names[mem[i].kernel]}:{mem[i].stmt}" for i in range(begin[g], begin[g + 1])]
                 for g in range(ng.value)]
+
+    def plan_search_ex(self, generations=30, population=24, seed=1, objective="model",
+                       max_group_kernels=0, reps=0, c_violation=0.0, c_sm=0.0, stream=None):
+        """Lazy-fission plan search (sp_plan_search_ex): objective "model" (host) or
+        "measured" (groups JIT-compiled and timed on the current device; arrays must be
+        bound).  Returns (plan, report dict)."""
+        o = SpSearchOptions(generations=int(generations), population=int(population),
+                            seed=int(seed), objective={"model": 0, "measured": 1}[objective],
+                            max_group_kernels=int(max_group_kernels), reps=int(reps),
+                            c_violation=float(c_violation), c_sm=float(c_sm))
+        rep = SpSearchReport()
+        ng = ctypes.c_int32()
+        nst = sum(len(k["stmts"]) for k in self.prog["kernels"])
+        begin = (ctypes.c_int32 * (nst + 1))()
+        mem = (SpStmtRef * nst)()
+        sh = _stream_handle(stream) if objective == "measured" else None
+        _check(lib().sp_plan_search_ex(self.handle, ctypes.byref(o), sh, nst, ctypes.byref(ng), begin, mem,
+                                       ctypes.byref(rep)))
+        names = [k["name"] for k in self.prog["kernels"]]
+        plan = [[f"{names[mem[i].kernel]}:{mem[i].stmt}" for i in range(begin[g], begin[g + 1])]
+                for g in range(ng.value)]
+        return plan, {f: getattr(rep, f) for f, _ in SpSearchReport._fields_}
 
     def n_launches(self, mode):
         n = ctypes.c_int32()

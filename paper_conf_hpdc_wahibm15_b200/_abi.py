@@ -56,6 +56,19 @@ class SpTileConfig(ctypes.Structure):
                                               "block_x", "block_y", "block_cby", "zqueue")]
 
 
+class SpSearchOptions(ctypes.Structure):
+    _fields_ = [("generations", ctypes.c_int32), ("population", ctypes.c_int32),
+                ("seed", ctypes.c_uint64), ("objective", ctypes.c_int32),
+                ("max_group_kernels", ctypes.c_int32), ("reps", ctypes.c_int32),
+                ("c_violation", ctypes.c_double), ("c_sm", ctypes.c_double)]
+
+
+class SpSearchReport(ctypes.Structure):
+    _fields_ = [("cost_us", ctypes.c_double), ("dp_cost_us", ctypes.c_double),
+                ("unfused_cost_us", ctypes.c_double), ("groups_evaluated", ctypes.c_int32),
+                ("fissioned_kernels", ctypes.c_int32), ("generations_run", ctypes.c_int32)]
+
+
 class SpEdge(ctypes.Structure):
     _fields_ = [("frm", ctypes.c_int32), ("to", ctypes.c_int32), ("kind", ctypes.c_int32),
                 ("array", ctypes.c_int32)]
@@ -85,7 +98,7 @@ EXPORTS = [
     "sp_signal_buffer", "sp_bind_peer", "sp_bind_peer_signal", "sp_ipc_export", "sp_ipc_open", "stencil_program_create",
     "stencil_program_destroy", "stencil_program_layout", "stencil_program_bind",
     "sp_program_set_option", "sp_program_counts", "sp_program_edges", "sp_fission_components",
-    "fusion_plan_set", "sp_plan_greedy", "sp_plan_search", "sp_plan_count", "sp_plan_report", "fusion_plan_report", "sp_plan_source",
+    "fusion_plan_set", "sp_plan_greedy", "sp_plan_search", "sp_plan_search_ex", "sp_plan_count", "sp_plan_report", "fusion_plan_report", "sp_plan_source",
     "sp_plan_exchange", "sp_plan_wave_offsets", "sp_plan_tune", "sp_compile", "sp_load", "run_unfused", "run_fused", "sp_run_launch", "sp_run_launch_count", "exchange_halos", "sp_last_error",
 ]
 
@@ -121,6 +134,8 @@ def lib():
             "sp_plan_count": [vp, i32, P(i32)],
             "sp_plan_greedy": [vp, i32, P(i32), P(i32), P(SpStmtRef)],
             "sp_plan_search": [vp, i32, i32, ctypes.c_uint64, i32, P(i32), P(i32), P(SpStmtRef)],
+            "sp_plan_search_ex": [vp, P(SpSearchOptions), vp, i32, P(i32), P(i32), P(SpStmtRef),
+                                  P(SpSearchReport)],
             "sp_plan_report": [vp, i32, i32, P(SpGroupReport)],
             "fusion_plan_report": [vp, i32, P(SpGroupReport)],
             "sp_plan_source": [vp, i32, ctypes.c_char_p, ctypes.c_size_t, P(ctypes.c_size_t)],

@@ -42,6 +42,8 @@ def _run(cmd):
 
 
 def embed_header():
+    """csrc/sf_device_embed.inc: the device header as a C++ raw string (the NVRTC header of
+    every generated kernel).  Generated here at every build, never edited or tracked."""
     src = open(os.path.join(CSRC, "device", "sf_device.cuh")).read()
     out = os.path.join(CSRC, "sf_device_embed.inc")
     text = 'R"SFDEV(' + src + ')SFDEV"\n'

@@ -419,6 +419,7 @@ sp_status sp_program_set_option(stencil_program *p, const char *key, int64_t v) 
         else if (k == "zwave_streams") o.zwave_streams = std::max(1, std::min(8, (int)v));
         else if (k == "xpush") o.xpush = v != 0;
         else if (k == "fastpath") o.fastpath = v != 0;
+        else if (k == "minblocks") o.minblocks = (int)std::max<int64_t>(1, std::min<int64_t>(v, 32));
         else if (k == "regcap") o.regcap = (int)std::min<int64_t>(v, 2);
         else if (k == "l2_flush") {}
         else fail(SP_E_ARG, "unknown option '" + k + "'");
@@ -503,8 +504,23 @@ sp_status sp_plan_search(stencil_program *p, int32_t generations, int32_t popula
                          int32_t cap, int32_t *n_groups, int32_t *group_begin, sp_stmt_ref *members) {
     return guard([&] {
         if (!p || !n_groups || generations < 0 || population < 1) fail(SP_E_ARG, "bad argument");
-        write_plan(p, search_plan(p, generations, population, seed), cap, n_groups, group_begin,
-                   members);
+        sp_search_options o;
+        std::memset(&o, 0, sizeof o);
+        o.generations = generations;
+        o.population = population;
+        o.seed = seed;
+        write_plan(p, search_plan(p, o, nullptr, nullptr), cap, n_groups, group_begin, members);
+    });
+}
+
+sp_status sp_plan_search_ex(stencil_program *p, const sp_search_options *opts, sp_stream stream,
+                            int32_t cap, int32_t *n_groups, int32_t *group_begin, sp_stmt_ref *members,
+                            sp_search_report *report) {
+    return guard([&] {
+        if (!p || !opts || !n_groups || opts->generations < 0 || opts->population < 0 ||
+            opts->objective < 0 || opts->objective > 1)
+            fail(SP_E_ARG, "bad argument");
+        write_plan(p, search_plan(p, *opts, stream, report), cap, n_groups, group_begin, members);
     });
 }
 

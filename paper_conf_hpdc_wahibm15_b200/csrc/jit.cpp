@@ -224,7 +224,8 @@ void compile_mode(stencil_program *p, Mode &m) {
                         // __launch_bounds__ overrides --maxrregcount and ptxas does not
                         // model the per-sub-partition limit: state the budget directly
                         std::string src2 = L.source;
-                        const std::string lb = "__launch_bounds__(" + std::to_string(L.nth) + ", 1)";
+                        const std::string lb = "__launch_bounds__(" + std::to_string(L.nth) + ", " +
+                                               std::to_string(std::max(1, p->opt.minblocks)) + ")";
                         const size_t at = src2.find(lb);
                         if (at != std::string::npos)
                             src2.replace(at, lb.size(), "__maxnreg__(" + std::to_string(cap) + ")");

@@ -24,8 +24,8 @@ namespace sf {
 static int64_t rup(int64_t v, int64_t m) { return (v + m - 1) / m * m; }
 
 // ----------------------------------------------------------------- analysis
-static Launch analyze_group(const stencil_program *p, const std::vector<int> &members,
-                            const std::set<int> &stored_gids) {
+Launch analyze_group(const stencil_program *p, const std::vector<int> &members,
+                     const std::set<int> &stored_gids) {
     Launch L;
     L.members = members;
     const int n = (int)members.size();
@@ -319,7 +319,7 @@ static double estimate_instr(const Launch &L, bool factor) {
 }
 
 // per-point byte/flop model of a configured launch
-static void model(const stencil_program *p, Launch &L) {
+void model(const stencil_program *p, Launch &L) {
     const int e = p->elem;
     const double tile = (double)L.tx * L.ty * L.zc;
     int n_store = 0;
@@ -367,7 +367,7 @@ static int max_region_points(const Launch &L) {
     return m;
 }
 
-static void choose_config(const stencil_program *p, Launch &L, bool quick = false) {
+void choose_config(const stencil_program *p, Launch &L, bool quick) {
     const sp_grid &g = p->grid;
     const int e = p->elem;
     const int64_t nz = g.nz_local;
@@ -486,8 +486,8 @@ static void choose_config(const stencil_program *p, Launch &L, bool quick = fals
 }
 
 // ---------------------------------------------------------------- plans
-static void live_out(const stencil_program *p, bool fused,
-                     const std::vector<std::vector<int>> &groups, std::vector<std::set<int>> &stored) {
+void live_out(const stencil_program *p, bool fused, const std::vector<std::vector<int>> &groups,
+              std::vector<std::set<int>> &stored) {
     stored.assign(groups.size(), {});
     const int na = (int)p->arrays.size();
     if (!fused) {
@@ -694,7 +694,7 @@ void sf_plan_set_impl(stencil_program *p, int32_t n_groups, const int32_t *group
 // group that violates a hazard (R11) or fits no tile is infeasible.
 namespace sf {
 // units of the plan search: fission pieces (§4.1) in program order
-static std::vector<std::vector<int>> fission_units(const stencil_program *p) {
+std::vector<std::vector<int>> fission_units(const stencil_program *p) {
     std::vector<std::vector<int>> units;
     for (size_t k = 0; k < p->kernels.size(); ++k) {
         int nc = 0;
@@ -766,171 +766,6 @@ std::vector<std::vector<int>> greedy_plan(stencil_program *p) {
     return groups;
 }
 
-// GGA-lite plan search (NEXT #1; the paper's grouping genetic algorithm
-// §3.2.4/§4, whose encoding and operators [27]/[28] the paper does not give, so this
-// is a plain grouping GA): a chromosome assigns every fission unit a group label;
-// it decodes to the groups in a topological order of the quotient of the unit
-// dependency DAG (ties: smallest unit first) and is illegal if the quotient has a
-// cycle (non-convex grouping) or a group fails analysis (hazard R11, no tile fits
-// in shared memory: the paper's smem-capacity penalty).  Units may be grouped out
-// of program order (independent statements reorder, P:L136 OEG).  Operators:
-// group-injection crossover (groups of one parent overwrite the other's labels),
-// merge of two groups, split of a group at a program-order cut, move of one unit to
-// a neighbour's group.  The population is seeded with the greedy plan, full
-// fission and one group per kernel; tournament selection with elitism.  The
-// objective is the plan cost model above (greedy_plan's); deterministic for a seed.
-std::vector<std::vector<int>> search_plan(stencil_program *p, int generations, int population,
-                                          uint64_t seed) {
-    const std::vector<std::vector<int>> units = fission_units(p);
-    const int nu = (int)units.size();
-    std::vector<int> unit_of(p->stmts.size(), -1);
-    for (int u = 0; u < nu; ++u)
-        for (int gid : units[u]) unit_of[gid] = u;
-    std::vector<std::vector<int>> succ(nu);
-    for (const sp_edge &e : p->edges) {
-        const int a = unit_of[e.from], b = unit_of[e.to];
-        if (a != b) succ[a].push_back(b);
-    }
-    for (auto &v : succ) {
-        std::sort(v.begin(), v.end());
-        v.erase(std::unique(v.begin(), v.end()), v.end());
-    }
-    uint64_t rs = seed * 0x9E3779B97F4A7C15ull + 0x632BE59BD9B4E019ull;
-    auto rnd = [&](int n) {  // splitmix64
-        rs += 0x9E3779B97F4A7C15ull;
-        uint64_t z = rs;
-        z = (z ^ (z >> 30)) * 0xBF58476D1CE4E5B9ull;
-        z = (z ^ (z >> 27)) * 0x94D049BB133111EBull;
-        return (int)((z ^ (z >> 31)) % (uint64_t)std::max(n, 1));
-    };
-    using Chrom = std::vector<int>;
-    auto normalize = [&](Chrom &c) {
-        std::map<int, int> ren;
-        for (int &l : c) {
-            auto it = ren.find(l);
-            if (it == ren.end()) it = ren.emplace(l, (int)ren.size()).first;
-            l = it->second;
-        }
-    };
-    auto decode = [&](const Chrom &c, std::vector<std::vector<int>> &gs) {
-        const int ng = *std::max_element(c.begin(), c.end()) + 1;
-        std::vector<std::vector<int>> mem(ng);
-        for (int u = 0; u < nu; ++u) mem[c[u]].push_back(u);
-        std::vector<std::set<int>> gsucc(ng);
-        std::vector<int> indeg(ng, 0);
-        for (int u = 0; u < nu; ++u)
-            for (int v : succ[u])
-                if (c[u] != c[v] && gsucc[c[u]].insert(c[v]).second) indeg[c[v]]++;
-        std::set<std::pair<int, int>> ready;  // (first unit, group)
-        for (int g = 0; g < ng; ++g)
-            if (!indeg[g] && !mem[g].empty()) ready.insert({mem[g][0], g});
-        gs.clear();
-        while (!ready.empty()) {
-            const int g = ready.begin()->second;
-            ready.erase(ready.begin());
-            std::vector<int> gids;
-            for (int u : mem[g]) gids.insert(gids.end(), units[u].begin(), units[u].end());
-            std::sort(gids.begin(), gids.end());
-            gs.push_back(gids);
-            for (int h : gsucc[g])
-                if (--indeg[h] == 0) ready.insert({mem[h][0], h});
-        }
-        int nonempty = 0;
-        for (auto &m : mem) nonempty += !m.empty();
-        return (int)gs.size() == nonempty;  // false: the quotient has a cycle
-    };
-    PlanCost pc{p, {}};
-    auto fitness = [&](const Chrom &c) {
-        std::vector<std::vector<int>> gs;
-        if (!decode(c, gs)) return 1e30;
-        return pc.plan(gs);
-    };
-    auto from_groups = [&](const std::vector<std::vector<int>> &gs) {
-        Chrom c(nu, 0);
-        for (size_t g = 0; g < gs.size(); ++g)
-            for (int gid : gs[g]) c[unit_of[gid]] = (int)g;
-        normalize(c);
-        return c;
-    };
-    auto mutate = [&](Chrom &c) {
-        const int ng = *std::max_element(c.begin(), c.end()) + 1;
-        const int op = rnd(3), u = rnd(nu);
-        if (op == 0) {  // merge u's group with the group of a program-order neighbour
-            const int v = std::min(nu - 1, std::max(0, u + (rnd(2) ? 1 : -1)));
-            const int a = c[u], b = c[v];
-            for (int &l : c)
-                if (l == b) l = a;
-        } else if (op == 1) {  // split u's group at a program-order cut
-            std::vector<int> mem;
-            for (int w = 0; w < nu; ++w)
-                if (c[w] == c[u]) mem.push_back(w);
-            if (mem.size() > 1) {
-                const int cut = 1 + rnd((int)mem.size() - 1);
-                for (size_t i = cut; i < mem.size(); ++i) c[mem[i]] = ng;
-            }
-        } else {  // move u to a neighbour's group
-            const int v = std::min(nu - 1, std::max(0, u + (rnd(2) ? 1 : -1)));
-            c[u] = c[v];
-        }
-        normalize(c);
-    };
-    auto crossover = [&](const Chrom &a, const Chrom &b) {
-        Chrom c = a;
-        int next = *std::max_element(a.begin(), a.end()) + 1;
-        const int ngb = *std::max_element(b.begin(), b.end()) + 1;
-        for (int g = 0; g < ngb; ++g) {
-            if (rnd(2)) continue;
-            for (int u = 0; u < nu; ++u)
-                if (b[u] == g) c[u] = next;
-            ++next;
-        }
-        normalize(c);
-        return c;
-    };
-    // initial population
-    std::vector<std::pair<double, Chrom>> pop;
-    auto add = [&](Chrom c) { pop.push_back({fitness(c), c}); };
-    const Chrom greedy = from_groups(greedy_plan(p));
-    add(greedy);
-    Chrom sep(nu);
-    for (int u = 0; u < nu; ++u) sep[u] = u;
-    add(sep);
-    Chrom perk(nu);
-    for (int u = 0; u < nu; ++u) perk[u] = p->stmts[units[u][0]].kernel;
-    normalize(perk);
-    add(perk);
-    while ((int)pop.size() < std::max(population, 4)) {
-        Chrom c = greedy;
-        for (int k = 1 + rnd(4); k > 0; --k) mutate(c);
-        add(c);
-    }
-    auto by_fit = [](const std::pair<double, Chrom> &x, const std::pair<double, Chrom> &y) {
-        return x.first < y.first || (x.first == y.first && x.second < y.second);
-    };
-    std::sort(pop.begin(), pop.end(), by_fit);
-    auto tournament = [&]() -> const Chrom & {
-        int best = rnd((int)pop.size());
-        for (int k = 0; k < 2; ++k) best = std::min(best, rnd((int)pop.size()));  // sorted: lower = fitter
-        return pop[best].second;
-    };
-    for (int gen = 0; gen < generations; ++gen) {
-        std::vector<std::pair<double, Chrom>> next(pop.begin(), pop.begin() + std::min<size_t>(2, pop.size()));
-        std::set<Chrom> seen;
-        for (auto &x : next) seen.insert(x.second);
-        int tries = 0;
-        while ((int)next.size() < (int)pop.size() && tries++ < 20 * (int)pop.size()) {
-            Chrom c = rnd(2) ? crossover(tournament(), tournament()) : tournament();
-            for (int k = 1 + rnd(2); k > 0; --k) mutate(c);
-            if (!seen.insert(c).second) continue;
-            next.push_back({fitness(c), c});
-        }
-        std::sort(next.begin(), next.end(), by_fit);
-        pop.swap(next);
-    }
-    std::vector<std::vector<int>> gs;
-    decode(pop.front().second, gs);
-    return gs;
-}
 }  // namespace sf
 
 void sf_unfused_prepare(stencil_program *p) {

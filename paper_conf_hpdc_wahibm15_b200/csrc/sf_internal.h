@@ -11,6 +11,7 @@
 #include <map>
 #include <memory>
 #include <mutex>
+#include <set>
 #include <string>
 #include <vector>
 
@@ -46,7 +47,10 @@ struct Options {
     int zwave = 0;          // z-wave schedule: planes per wave (0 = one launch per group per step)
     int zwave_streams = 2;  // waves in flight (streams) of the z-wave schedule
     int xpush = 0;  // several ranks: stores push in-step halo planes into the neighbours' ghosts
-    int fastpath = 1;  // emit a predicate-free step body for interior tiles / planes
+    int fastpath = 0;  // emit a second, predicate-free step body for interior tiles / planes
+                       // (r2: 40 % fewer issued instructions per step, but the doubled code
+                       // overflows the 32 KB instruction cache: C4 +2 %, C2 +12 % slower)
+    int minblocks = 1; // __launch_bounds__ minimum resident CTAs (register budget for ptxas)
     int regcap = 1; // recompile a few registers tighter when that adds a resident CTA:
                     // 0 never, 1 peer-push kernels, 2 every kernel
 };
@@ -206,8 +210,17 @@ void analyze_mode(stencil_program *p, bool fused, const std::vector<std::vector<
                   Mode &out);
 void fill_report(const stencil_program *p, const Launch &L, sp_group_report *r);
 std::vector<std::vector<int>> greedy_plan(stencil_program *p);
-std::vector<std::vector<int>> search_plan(stencil_program *p, int generations, int population,
-                                          uint64_t seed);
+Launch analyze_group(const stencil_program *p, const std::vector<int> &members,
+                     const std::set<int> &stored_gids);
+void choose_config(const stencil_program *p, Launch &L, bool quick = false);
+void model(const stencil_program *p, Launch &L);
+void live_out(const stencil_program *p, bool fused, const std::vector<std::vector<int>> &groups,
+              std::vector<std::set<int>> &stored);
+std::vector<std::vector<int>> fission_units(const stencil_program *p);
+
+// search.cpp: lazy-fission plan search (NEXT #1)
+std::vector<std::vector<int>> search_plan(stencil_program *p, const sp_search_options &o, void *stream,
+                                          sp_search_report *rep);
 
 // codegen.cpp
 std::string generate_launch(const stencil_program *p, Launch &L, int index, bool fused);

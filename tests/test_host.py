@@ -546,3 +546,27 @@ def test_run_launch_count():
     recv = [i for i in range(len(plan)) if q.exchange_plan("fused", i)]
     assert recv
     assert q.launch_count("fused") == len(plan) + len(recv)
+
+
+def test_lazy_fission_search_model_objective():
+    """sp_plan_search_ex (NEXT #1) with the model objective: deterministic,
+    legal, never worse than its exact contiguous-segmentation DP seed, which is never
+    worse than the unfused plan; on C4 (no kernel needs fission) no kernel is split, on
+    C3 the search fissions K0's two independent outputs (P and Q, Fig.-3 style) and fuses
+    one of them with its consumer."""
+    from synth.scale_les import c4
+    for name, prog in (("C4", c4(nx=256, ny=32, nz=64)), ("C3", P.c3())):
+        p = Program(prog)
+        plan, rep = p.plan_search_ex(generations=15, population=12, seed=2)
+        assert (plan, rep) == p.plan_search_ex(generations=15, population=12, seed=2)
+        p.set_plan(plan)
+        refs = [r for g in plan for r in g]
+        assert len(refs) == len(set(refs)) == sum(len(k["stmts"]) for k in prog["kernels"])
+        assert rep["cost_us"] <= rep["dp_cost_us"] + 1e-9 <= rep["unfused_cost_us"] + 1e-9
+        assert rep["generations_run"] == 15 and rep["groups_evaluated"] > len(prog["kernels"])
+        if name == "C4":
+            assert rep["fissioned_kernels"] == 0
+        else:
+            assert rep["fissioned_kernels"] == 1
+            k0 = [g for g in plan if any(r.startswith("K0:") for r in g)]
+            assert len(k0) == 2 and any(len(g) > 1 for g in k0)

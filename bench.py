@@ -162,6 +162,14 @@ def run_ours(args):
     world = int(os.environ.get("WORLD_SIZE", "1"))
     rank = int(os.environ.get("RANK", "0"))
     local = int(os.environ.get("LOCAL_RANK", "0"))
+    if os.environ.get("SF_BENCH_SHARE_GPU") == "1" and world > 1:
+        # functional test of the N > 1 path on ONE GPU (tests/test_gpu_nccl.py): every rank
+        # on cuda:0, NCCL told the ranks sit on different hosts (socket transport over
+        # loopback); the numbers of such a run measure nothing and are labelled so
+        local = 0
+        os.environ.update({"NCCL_HOSTID": f"stencilfuse-rank{rank}", "NCCL_SOCKET_IFNAME": "lo",
+                           "NCCL_IB_DISABLE": "1", "NCCL_P2P_DISABLE": "1", "NCCL_SHM_DISABLE": "1",
+                           "NCCL_NVLS_ENABLE": "0"})
     if world > 1:
         torch.cuda.set_device(local)
         dist.init_process_group("nccl", device_id=torch.device("cuda", local))
@@ -394,6 +402,8 @@ def run_ours(args):
                        "halo_exchange": ("peer-push (TEMP) + NCCL (step-start)" if xpush else
                                          "NCCL send/recv") if world > 1 else "none",
                        "l2": "no flush: per-GPU working set > 126 MB L2"},
+            **({"functional_test": "SF_BENCH_SHARE_GPU=1: all ranks share one GPU; not a measurement"}
+               if os.environ.get("SF_BENCH_SHARE_GPU") == "1" else {}),
             "hbm_gbs_alg": alg_step / (step_ms * 1e-3) / 1e9,
             "roofline_step": {"achieved": alg_step / (step_ms * 1e-3) / 1e9, "peak": peak,
                               "unit": "GB/s", "frac": alg_step / (step_ms * 1e-3) / 1e9 / peak,
@@ -520,7 +530,7 @@ def ensure_world(args):
         return
     if args.gpus <= 1:
         return
-    if args.impl == "ours":
+    if args.impl == "ours" and os.environ.get("SF_BENCH_SHARE_GPU") != "1":
         import torch
         have = torch.cuda.device_count()
         if have < args.gpus:

@@ -269,6 +269,18 @@ sp_status fusion_plan_set(stencil_program *prog, int32_t n_groups, const int32_t
  * With group_begin == NULL only *n_groups is returned.  Does not set the plan. */
 sp_status sp_plan_greedy(stencil_program *prog, int32_t cap, int32_t *n_groups,
                          int32_t *group_begin, sp_stmt_ref *members);
+/* Launch configuration (0 = left to the model-driven chooser).  The thread
+ * geometry must satisfy tile_x = (tile_x/block_x)*block_x and
+ * tile_y = (threads/(tile_x/block_x)) * block_y * block_cby.
+ * zqueue selects how values read at several planes are kept across z steps:
+ * 0 = the program's "zqueue" option, 1 = shared-memory loads only, 2 = register
+ * queues per statement, 3 = step-wide register queues of the input columns a
+ * thread owns (results are bit-identical under every policy). */
+typedef struct {
+    int32_t tile_x, tile_y, zchunk, threads, prefetch, block_x, block_y, block_cby;
+    int32_t zqueue;
+} sp_tile_config;
+
 /* Lazy-fission plan search (the paper's search step,
  * P:L140 §3.2.4 and §4.1).  Steps:
  *   1. metadata pre-step: the objective is evaluated for every original kernel and
@@ -294,7 +306,11 @@ sp_status sp_plan_greedy(stencil_program *prog, int32_t cap, int32_t *n_groups,
  * on the current device with CUDA events on `stream` (median of `reps` launches,
  * L2 flushed before each; the paper's empirical metadata, §3.2.1); the
  * program's arrays must be bound, and their contents are overwritten.
- * Output as sp_plan_greedy; `report` (nullable) receives costs and counts. */
+ * With candidate configurations (measured objective) every group is also timed at
+ * each one that fits and costs its fastest; `configs` (nullable, >= cap entries,
+ * written with the groups) receives each returned group's configuration for
+ * sp_plan_tune (all zero: the chooser's).  Output as sp_plan_greedy; `report`
+ * (nullable) receives costs and counts. */
 typedef struct {
     int32_t generations;        /* GA generations (0: pre-step + DP + seeds only)            */
     int32_t population;         /* GA population (clamped to >= 4)                            */
@@ -304,6 +320,8 @@ typedef struct {
     int32_t reps;               /* measured: timed launches per group, median (0 -> 5)        */
     double c_violation;         /* C_i per violated constraint, x the unfused plan cost (0 -> 1) */
     double c_sm;                /* |C_SM|, x the unfused plan cost (0 -> 0.5)                  */
+    int32_t n_configs;          /* measured: candidate tile configurations timed per group    */
+    const sp_tile_config *configs; /* besides the chooser's; a group costs its fastest one    */
 } sp_search_options;
 typedef struct {
     double cost_us;             /* objective of the returned plan                             */
@@ -315,7 +333,7 @@ typedef struct {
 } sp_search_report;
 sp_status sp_plan_search_ex(stencil_program *prog, const sp_search_options *opts, sp_stream stream,
                             int32_t cap, int32_t *n_groups, int32_t *group_begin, sp_stmt_ref *members,
-                            sp_search_report *report);
+                            sp_tile_config *configs, sp_search_report *report);
 /* sp_plan_search_ex with the model objective and default constants.  Host-only. */
 sp_status sp_plan_search(stencil_program *prog, int32_t generations, int32_t population, uint64_t seed,
                          int32_t cap, int32_t *n_groups, int32_t *group_begin, sp_stmt_ref *members);
@@ -327,17 +345,6 @@ sp_status sp_plan_report(const stencil_program *prog, int32_t mode, int32_t laun
 sp_status fusion_plan_report(const stencil_program *prog, int32_t group, sp_group_report *out);
 /* Generated CUDA source of a mode (for inspection); *len receives the full size. */
 sp_status sp_plan_source(stencil_program *prog, int32_t mode, char *buf, size_t cap, size_t *len);
-/* Launch configuration (0 = left to the model-driven chooser).  The thread
- * geometry must satisfy tile_x = (tile_x/block_x)*block_x and
- * tile_y = (threads/(tile_x/block_x)) * block_y * block_cby.
- * zqueue selects how values read at several planes are kept across z steps:
- * 0 = the program's "zqueue" option, 1 = shared-memory loads only, 2 = register
- * queues per statement, 3 = step-wide register queues of the input columns a
- * thread owns (results are bit-identical under every policy). */
-typedef struct {
-    int32_t tile_x, tile_y, zchunk, threads, prefetch, block_x, block_y, block_cby;
-    int32_t zqueue;
-} sp_tile_config;
 
 /* Empirical tuning hook (the paper's per-kernel block-size tuning, §4.2):
  * pin the configuration of one launch of a mode; cfg == NULL removes the pin.

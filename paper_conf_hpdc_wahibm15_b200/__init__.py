@@ -322,26 +322,38 @@ class Program:
                 for g in range(ng.value)]
 
     def plan_search_ex(self, generations=30, population=24, seed=1, objective="model",
-                       max_group_kernels=0, reps=0, c_violation=0.0, c_sm=0.0, stream=None):
+                       max_group_kernels=0, reps=0, c_violation=0.0, c_sm=0.0, configs=None,
+                       stream=None, with_configs=False):
         """Lazy-fission plan search (sp_plan_search_ex): objective "model" (host) or
-        "measured" (groups JIT-compiled and timed on the current device; arrays must be
-        bound).  Returns (plan, report dict)."""
+        "measured" (groups JIT-compiled and timed on the current device at the chooser's
+        and each candidate configuration in `configs`; arrays must be bound).  Returns
+        (plan, report dict) or, with_configs, (plan, per-group configuration dicts, report)."""
+        cands = [SpTileConfig(**{k: int(v) for k, v in c.items() if k in dict(SpTileConfig._fields_)})
+                 for c in (configs or [])]
+        carr = (SpTileConfig * max(1, len(cands)))(*cands)
         o = SpSearchOptions(generations=int(generations), population=int(population),
                             seed=int(seed), objective={"model": 0, "measured": 1}[objective],
                             max_group_kernels=int(max_group_kernels), reps=int(reps),
-                            c_violation=float(c_violation), c_sm=float(c_sm))
+                            c_violation=float(c_violation), c_sm=float(c_sm),
+                            n_configs=len(cands), configs=carr)
         rep = SpSearchReport()
         ng = ctypes.c_int32()
         nst = sum(len(k["stmts"]) for k in self.prog["kernels"])
         begin = (ctypes.c_int32 * (nst + 1))()
         mem = (SpStmtRef * nst)()
+        out_cfg = (SpTileConfig * nst)()
         sh = _stream_handle(stream) if objective == "measured" else None
         _check(lib().sp_plan_search_ex(self.handle, ctypes.byref(o), sh, nst, ctypes.byref(ng), begin, mem,
-                                       ctypes.byref(rep)))
+                                       out_cfg, ctypes.byref(rep)))
         names = [k["name"] for k in self.prog["kernels"]]
         plan = [[f"{names[mem[i].kernel]}:{mem[i].stmt}" for i in range(begin[g], begin[g + 1])]
                 for g in range(ng.value)]
-        return plan, {f: getattr(rep, f) for f, _ in SpSearchReport._fields_}
+        report = {f: getattr(rep, f) for f, _ in SpSearchReport._fields_}
+        if not with_configs:
+            return plan, report
+        cfgs = [{f: getattr(out_cfg[g], f) for f, _ in SpTileConfig._fields_ if getattr(out_cfg[g], f)}
+                or None for g in range(ng.value)]
+        return plan, cfgs, report
 
     def n_launches(self, mode):
         n = ctypes.c_int32()

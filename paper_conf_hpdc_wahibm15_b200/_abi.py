@@ -60,7 +60,8 @@ class SpSearchOptions(ctypes.Structure):
     _fields_ = [("generations", ctypes.c_int32), ("population", ctypes.c_int32),
                 ("seed", ctypes.c_uint64), ("objective", ctypes.c_int32),
                 ("max_group_kernels", ctypes.c_int32), ("reps", ctypes.c_int32),
-                ("c_violation", ctypes.c_double), ("c_sm", ctypes.c_double)]
+                ("c_violation", ctypes.c_double), ("c_sm", ctypes.c_double),
+                ("n_configs", ctypes.c_int32), ("configs", ctypes.POINTER(SpTileConfig))]
 
 
 class SpSearchReport(ctypes.Structure):
@@ -135,7 +136,7 @@ def lib():
             "sp_plan_greedy": [vp, i32, P(i32), P(i32), P(SpStmtRef)],
             "sp_plan_search": [vp, i32, i32, ctypes.c_uint64, i32, P(i32), P(i32), P(SpStmtRef)],
             "sp_plan_search_ex": [vp, P(SpSearchOptions), vp, i32, P(i32), P(i32), P(SpStmtRef),
-                                  P(SpSearchReport)],
+                                  P(SpTileConfig), P(SpSearchReport)],
             "sp_plan_report": [vp, i32, i32, P(SpGroupReport)],
             "fusion_plan_report": [vp, i32, P(SpGroupReport)],
             "sp_plan_source": [vp, i32, ctypes.c_char_p, ctypes.c_size_t, P(ctypes.c_size_t)],

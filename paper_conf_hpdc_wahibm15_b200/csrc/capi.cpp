@@ -509,18 +509,23 @@ sp_status sp_plan_search(stencil_program *p, int32_t generations, int32_t popula
         o.generations = generations;
         o.population = population;
         o.seed = seed;
-        write_plan(p, search_plan(p, o, nullptr, nullptr), cap, n_groups, group_begin, members);
+        write_plan(p, search_plan(p, o, nullptr, nullptr, nullptr), cap, n_groups, group_begin, members);
     });
 }
 
 sp_status sp_plan_search_ex(stencil_program *p, const sp_search_options *opts, sp_stream stream,
                             int32_t cap, int32_t *n_groups, int32_t *group_begin, sp_stmt_ref *members,
-                            sp_search_report *report) {
+                            sp_tile_config *configs, sp_search_report *report) {
     return guard([&] {
         if (!p || !opts || !n_groups || opts->generations < 0 || opts->population < 0 ||
-            opts->objective < 0 || opts->objective > 1)
+            opts->objective < 0 || opts->objective > 1 || opts->n_configs < 0 ||
+            (opts->n_configs > 0 && !opts->configs))
             fail(SP_E_ARG, "bad argument");
-        write_plan(p, search_plan(p, *opts, stream, report), cap, n_groups, group_begin, members);
+        std::vector<sp_tile_config> cfgs;
+        const auto gs = search_plan(p, *opts, stream, report, &cfgs);
+        write_plan(p, gs, cap, n_groups, group_begin, members);
+        if (configs && group_begin)
+            for (size_t g = 0; g < gs.size(); ++g) configs[g] = cfgs[g];
     });
 }
 

@@ -359,24 +359,12 @@ std::string generate_launch(const stencil_program *p, Launch &L, int index, bool
             l2_prefetch("j", "        ");
             o << "      }\n";
         }
-        // first batch: every input's planes [qlo, KF + ahi]; then one plane (j + ahi) of
-        // every input per step, a constant byte count (compact producer code: its loop
-        // shares the SM's instruction cache with the compute warps)
-        o << "      {\n        const int j = KF;\n";
-        if (L2PF > 0) l2_prefetch("(j + " + num(L2PF) + ")", "        ");
-        batch(o, "        ");
-        o << "      }\n";
-        int64_t steady = 0;
-        for (int a = 0; a < nin; ++a) steady += box_bytes(a);
-        o << "      for (int j = KF + 1; j < zc; ++j) {\n";
+        o << "      for (int j = KF; j < zc; ++j) {\n";
         if (L2PF > 0) l2_prefetch("(j + " + num(L2PF) + ")", "        ");
         o << "        const int s = j - 1 - PF;  // step whose slots batch j overwrites\n";
         o << "        if (s >= KF) sf_mbar_wait(&empty[(s - KF) & " << NE - 1 << "], ((s - KF) >> "
           << log2i(NE) << ") & 1);\n";
-        o << "        sf_u64 *bar = &full[(j - KF) & " << NB - 1 << "];\n";
-        o << "        sf_mbar_expect_tx(bar, " << steady << "u);\n";
-        for (int a = 0; a < nin; ++a)
-            o << "        { const int q = j + (" << L.in[a].ahi << "); " << issue_plane(a) << " }\n";
+        batch(o, "        ");
         o << "      }\n    }\n    return;\n  }\n";
     }
     // compute warps store arrays the previous group may still read (WAR) and read

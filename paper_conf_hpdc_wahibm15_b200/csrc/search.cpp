@@ -55,25 +55,49 @@ class Objective {
         return it->second;
     }
     int evaluated() const { return (int)cache_.size(); }
+    // configuration the objective's time was obtained with (zeros: the chooser's)
+    sp_tile_config config(const Key &k) const {
+        auto it = cfg_.find(k);
+        if (it != cfg_.end()) return it->second;
+        sp_tile_config c;
+        std::memset(&c, 0, sizeof c);
+        return c;
+    }
 
   protected:
     virtual void evaluate(const std::vector<Key> &todo) = 0;
-    // group analysis + tile choice; false (with e.viol set) if the group is illegal
-    bool configure(const Key &k, Launch &L, Eval &e, bool quick) {
+    // group analysis + tile choice (pinned to `pin` when given, as sp_plan_tune does);
+    // false (with e.viol set) if the group is illegal or the pin does not fit
+    bool configure(const Key &k, Launch &L, Eval &e, bool quick, const sp_tile_config *pin = nullptr) {
         const std::set<int> st(k.second.begin(), k.second.end());
+        const Options saved = p_->opt;
         try {
             L = analyze_group(p_, k.first, st);
             if (L.dead) return false;
+            if (pin) {
+                if (pin->tile_x) p_->opt.tile_x = pin->tile_x;
+                if (pin->tile_y) p_->opt.tile_y = pin->tile_y;
+                if (pin->zchunk) p_->opt.zchunk = pin->zchunk;
+                if (pin->threads) p_->opt.threads = pin->threads;
+                if (pin->prefetch) p_->opt.prefetch = pin->prefetch;
+                if (pin->block_x) p_->opt.block_x = pin->block_x;
+                if (pin->block_y) p_->opt.block_y = pin->block_y;
+                if (pin->block_cby) p_->opt.block_cby = pin->block_cby;
+                if (pin->zqueue) p_->opt.zqueue = pin->zqueue - 1;
+            }
             choose_config(p_, L, quick);
+            p_->opt = saved;
             model(p_, L);
             return true;
         } catch (const Error &er) {
+            p_->opt = saved;
             e.viol = er.code == SP_E_PLAN_HAZARD ? 1 : 2;
             return false;
         }
     }
     stencil_program *p_;
     std::map<Key, Eval> cache_;
+    std::map<Key, sp_tile_config> cfg_;
 };
 
 // the library's launch-time model (plan.cpp::choose_config), + 3 us per launch
@@ -92,13 +116,16 @@ class ModelObjective : public Objective {
     }
 };
 
-// measured on the device: every new group of a batch is generated, JIT-compiled
-// (in parallel), loaded and timed with CUDA events on the caller's stream — median
-// of `reps` launches, each after a 256 MB memset that evicts the L2
+// measured on the device: every new group of a batch is generated at the chooser's
+// configuration and at each candidate configuration that fits, JIT-compiled (in
+// parallel), loaded and timed with CUDA events on the caller's stream — median of
+// `reps` launches, each after a 256 MB memset that evicts the L2; a group's time is
+// its fastest configuration (the paper's per-kernel block tuning, §4.2, folded
+// into the objective), remembered for the returned plan
 class MeasuredObjective : public Objective {
   public:
-    MeasuredObjective(stencil_program *p, void *stream, int reps)
-        : Objective(p), stream_((cudaStream_t)stream), reps_(std::max(1, reps)) {}
+    MeasuredObjective(stencil_program *p, void *stream, int reps, std::vector<sp_tile_config> cands)
+        : Objective(p), stream_((cudaStream_t)stream), reps_(std::max(1, reps)), cands_(std::move(cands)) {}
     ~MeasuredObjective() override {
         if (flush_) cudaFree(flush_);
         if (ev_[0]) cudaEventDestroy(ev_[0]);
@@ -109,18 +136,33 @@ class MeasuredObjective : public Objective {
     void evaluate(const std::vector<Key> &todo) override {
         ensure_cuda();
         Mode m;
-        std::vector<size_t> owner;
+        std::vector<std::pair<size_t, sp_tile_config>> owner;  // (key index, configuration)
         for (size_t i = 0; i < todo.size(); ++i) {
             Eval e;
-            Launch L;
-            if (!configure(todo[i], L, e, false)) {
-                cache_[todo[i]] = e;
-                continue;
+            bool any = false;
+            for (int v = -1; v < (int)cands_.size(); ++v) {
+                Launch L;
+                Eval ev;
+                if (!configure(todo[i], L, ev, false, v < 0 ? nullptr : &cands_[v])) {
+                    if (v < 0) e = ev;  // the chooser's verdict (hazard / no tile fits)
+                    if (v < 0 && (ev.viol || L.dead)) break;
+                    continue;
+                }
+                sp_tile_config c;
+                std::memset(&c, 0, sizeof c);
+                c.tile_x = L.tx; c.tile_y = L.ty; c.zchunk = L.zc; c.threads = L.nt; c.prefetch = L.pf;
+                c.block_x = L.vx; c.block_y = L.vy; c.block_cby = L.cby;
+                bool dup = false;
+                for (const auto &o : owner)
+                    dup |= o.first == i && !std::memcmp(&o.second, &c, sizeof c);
+                if (dup) continue;
+                L.name = "search" + std::to_string(i);
+                generate_launch(p_, L, (int)m.launches.size(), true);
+                m.launches.push_back(std::move(L));
+                owner.push_back({i, c});
+                any = true;
             }
-            L.name = "search" + std::to_string(i);
-            generate_launch(p_, L, (int)m.launches.size(), true);
-            m.launches.push_back(std::move(L));
-            owner.push_back(i);
+            if (!any) cache_[todo[i]] = e;
         }
         if (m.launches.empty()) return;
         m.analyzed = true;
@@ -134,22 +176,32 @@ class MeasuredObjective : public Objective {
         for (size_t j = 0; j < m.launches.size(); ++j) {
             launch(p_, m, (int)j, stream_);  // first use (module, descriptors)
             std::vector<float> ts;
+            auto ck = [&](cudaError_t e, const char *what) {
+                if (e != cudaSuccess)
+                    fail(SP_E_CUDA, std::string("search: ") + what + " (" + m.launches[j].fn + ", tile " +
+                                        std::to_string(m.launches[j].tx) + "x" + std::to_string(m.launches[j].ty) +
+                                        "): " + cudaGetErrorString(e));
+            };
             for (int r = 0; r < reps_; ++r) {
                 float ms = 0;
-                if (cudaMemsetAsync(flush_, r & 0xff, kFlush, stream_) != cudaSuccess ||
-                    cudaEventRecord(ev_[0], stream_) != cudaSuccess)
-                    fail(SP_E_CUDA, "search: timing");
+                ck(cudaMemsetAsync(flush_, r & 0xff, kFlush, stream_), "L2 flush");
+                ck(cudaEventRecord(ev_[0], stream_), "event record");
                 launch(p_, m, (int)j, stream_);
-                if (cudaEventRecord(ev_[1], stream_) != cudaSuccess ||
-                    cudaEventSynchronize(ev_[1]) != cudaSuccess ||
-                    cudaEventElapsedTime(&ms, ev_[0], ev_[1]) != cudaSuccess)
-                    fail(SP_E_CUDA, "search: timing");
+                ck(cudaEventRecord(ev_[1], stream_), "event record");
+                ck(cudaEventSynchronize(ev_[1]), "kernel");
+                ck(cudaEventElapsedTime(&ms, ev_[0], ev_[1]), "elapsed");
                 ts.push_back(ms);
             }
             std::sort(ts.begin(), ts.end());
-            Eval e;
-            e.t = ts[ts.size() / 2] * 1e-3;
-            cache_[todo[owner[j]]] = e;
+            const double t = ts[ts.size() / 2] * 1e-3;
+            const Key &k = todo[owner[j].first];
+            auto it = cache_.find(k);
+            if (it == cache_.end() || t < it->second.t) {
+                Eval e;
+                e.t = t;
+                cache_[k] = e;
+                cfg_[k] = owner[j].second;
+            }
         }
         unload_mode(m);
     }
@@ -158,6 +210,7 @@ class MeasuredObjective : public Objective {
     static constexpr size_t kFlush = 256u << 20;
     cudaStream_t stream_;
     int reps_;
+    std::vector<sp_tile_config> cands_;
     void *flush_ = nullptr;
     cudaEvent_t ev_[2] = {nullptr, nullptr};
 };
@@ -173,9 +226,11 @@ uint64_t splitmix(uint64_t &s) {
 }  // namespace
 
 std::vector<std::vector<int>> search_plan(stencil_program *p, const sp_search_options &opt, void *stream,
-                                          sp_search_report *rep) {
+                                          sp_search_report *rep, std::vector<sp_tile_config> *configs) {
     std::unique_ptr<Objective> obj;
-    if (opt.objective == 1) obj.reset(new MeasuredObjective(p, stream, opt.reps > 0 ? opt.reps : 5));
+    if (opt.objective == 1)
+        obj.reset(new MeasuredObjective(p, stream, opt.reps > 0 ? opt.reps : 5,
+                                        std::vector<sp_tile_config>(opt.configs, opt.configs + std::max(0, opt.n_configs))));
     else obj.reset(new ModelObjective(p));
     const int K = (int)p->kernels.size();
     const int U = opt.max_group_kernels > 0 ? opt.max_group_kernels : 8;
@@ -497,6 +552,10 @@ std::vector<std::vector<int>> search_plan(stencil_program *p, const sp_search_op
     }
     std::vector<std::vector<int>> gs;
     decode(pop.front().second, gs);
+    if (configs) {
+        configs->clear();
+        for (const Key &k : plan_keys(gs)) configs->push_back(obj->config(k));
+    }
     if (rep) {
         std::memset(rep, 0, sizeof(*rep));
         rep->cost_us = pop.front().first * 1e6;

@@ -220,7 +220,7 @@ std::vector<std::vector<int>> fission_units(const stencil_program *p);
 
 // search.cpp: lazy-fission plan search (NEXT #1)
 std::vector<std::vector<int>> search_plan(stencil_program *p, const sp_search_options &o, void *stream,
-                                          sp_search_report *rep);
+                                          sp_search_report *rep, std::vector<sp_tile_config> *configs);
 
 // codegen.cpp
 std::string generate_launch(const stencil_program *p, Launch &L, int index, bool fused);

@@ -58,3 +58,25 @@ def test_nccl_exchange_halos_and_runs_two_processes(cuda_device):
     out = _run_two_ranks(CASES)
     print("\n".join(out))
     assert len(out) == 1 + len(CASES)
+
+
+def test_bench_multirank_path_two_processes(cuda_device):
+    """bench.py --gpus 2 (the driver's multi-GPU launch: it re-executes itself under
+    torch.distributed.run) runs end to end on one GPU with SF_BENCH_SHARE_GPU=1 (both ranks
+    on cuda:0, NCCL across "hosts"): torch's NCCL process group, the library's NCCL halo
+    exchange inside run_fused, the max-over-ranks timing and the e2e leg; rank 0 prints one
+    JSON line with n_gpus 2, z-slab x2 and NCCL exchange.  C2 (small) keeps it quick."""
+    import json
+    import subprocess
+    import sys
+    root = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+    env = dict(os.environ, SF_BENCH_SHARE_GPU="1")
+    r = subprocess.run([sys.executable, os.path.join(root, "bench.py"), "--gpus", "2", "--steps", "3",
+                        "--warmup", "3", "--workload", "C2", "--no-cpu"], capture_output=True, text=True,
+                       timeout=900, env=env, cwd=root)
+    lines = [l for l in r.stdout.splitlines() if l.startswith("{")]
+    assert r.returncode == 0 and len(lines) == 1, r.stdout[-3000:] + r.stderr[-3000:]
+    d = json.loads(lines[0])
+    assert d["n_gpus"] == 2 and d["config"]["parallelism"] == "z-slab x2"
+    assert d["config"]["halo_exchange"] == "NCCL send/recv" and d["gpu_launches"] > 0
+    assert "functional_test" in d

@@ -1,0 +1,80 @@
+"""The library's own plan search on the device (sp_plan_search_ex, objective = measured):
+metadata pre-step, DP over contiguous kernel segments, lazy-fission GA with the dynamic
+penalty f_p; every candidate group timed at the tile chooser's configuration and at each
+CANDIDATES entry (a group costs its fastest).  Writes a plan file bench.py can load.
+
+python tools/search_plan.py C4 [--out configs/c4_plan_search.json] [--generations 12]
+                               [--population 16] [--seed 1]
+(bench: SF_C4_PLAN=<out> python bench.py)
+"""
+import argparse
+import json
+import os
+import sys
+import time
+
+ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+sys.path.insert(0, ROOT)
+
+# candidate launch configurations (tile_x, tile_y, threads, block_x, block_y, block_cby,
+# zchunk, prefetch): the shapes the r1/r2 in-context tuners pinned for the C2-C5 groups
+CANDIDATES = [
+    dict(tile_x=32, tile_y=16, threads=64, block_x=1, block_y=8, block_cby=1, zchunk=16, prefetch=2),
+    dict(tile_x=32, tile_y=8, threads=128, block_x=1, block_y=2, block_cby=1, zchunk=16, prefetch=3),
+    dict(tile_x=32, tile_y=8, threads=64, block_x=2, block_y=2, block_cby=1, zchunk=32, prefetch=1),
+    dict(tile_x=32, tile_y=16, threads=256, block_x=1, block_y=1, block_cby=2, zchunk=16, prefetch=2),
+    dict(tile_x=32, tile_y=32, threads=64, block_x=1, block_y=4, block_cby=4, zchunk=8, prefetch=3),
+    dict(tile_x=64, tile_y=4, threads=128, block_x=1, block_y=2, block_cby=1, zchunk=32, prefetch=3),
+    dict(tile_x=128, tile_y=2, threads=128, block_x=1, block_y=2, block_cby=1, zchunk=32, prefetch=3),
+    dict(tile_x=32, tile_y=16, threads=128, block_x=1, block_y=4, block_cby=1, zchunk=16, prefetch=2),
+    dict(tile_x=32, tile_y=16, threads=128, block_x=2, block_y=2, block_cby=1, zchunk=16, prefetch=3),
+    dict(tile_x=32, tile_y=8, threads=128, block_x=1, block_y=2, block_cby=1, zchunk=32, prefetch=2),
+]
+
+
+def measured_search(workload, generations=12, population=16, seed=1, candidates=CANDIDATES, reps=3):
+    """Run the search on a full-size instance of the workload; returns the plan-file dict."""
+    import torch
+    import bench
+    from paper_conf_hpdc_wahibm15_b200 import Program
+    prog = bench.load_workload(workload)
+    dev = torch.device("cuda:0")
+    p = Program(prog)
+    p.allocate(dev, fill=0.0)
+    bench.fill_inputs(p, prog, dev, 0, prog["grid"]["ghost"][2])
+    t0 = time.time()
+    plan, cfgs, rep = p.plan_search_ex(generations=generations, population=population, seed=seed,
+                                       objective="measured", reps=reps, configs=candidates,
+                                       with_configs=True)
+    out = {"workload": workload,
+           "planner": f"sp_plan_search_ex (objective=measured, generations {generations}, population "
+                      f"{population}, seed {seed}, {len(candidates)} candidate configurations; "
+                      f"tools/search_plan.py)",
+           "search_seconds": time.time() - t0, "search_report": rep, "groups": plan, "configs": cfgs}
+    if workload == "C4":  # the unfused baseline's per-kernel pins are plan independent
+        fz = json.load(open(os.path.join(ROOT, "configs", "c4_plan.json")))
+        out["unfused_configs"] = fz.get("unfused_configs")
+        out["unfused_tuner"] = fz.get("unfused_tuner")
+    del p
+    return out
+
+
+def main():
+    ap = argparse.ArgumentParser()
+    ap.add_argument("workload")
+    ap.add_argument("--out", default=None)
+    ap.add_argument("--generations", type=int, default=12)
+    ap.add_argument("--population", type=int, default=16)
+    ap.add_argument("--seed", type=int, default=1)
+    a = ap.parse_args()
+    out = measured_search(a.workload, a.generations, a.population, a.seed)
+    print(json.dumps(out["search_report"]), f"{out['search_seconds']:.0f} s")
+    for g, c in zip(out["groups"], out["configs"]):
+        print(g, c)
+    if a.out:
+        json.dump(out, open(a.out, "w"), indent=1)
+        print("wrote", a.out)
+
+
+if __name__ == "__main__":
+    main()

@@ -57,7 +57,7 @@ def c2_boxed(nz):
 
 
 @pytest.mark.parametrize("cfg,ranks", [("C2", 2), ("C5", 3), ("C3", 2), ("C4", 2), ("chain3", 3),
-                                       ("C2box", 2)])
+                                       ("C2box", 2), ("chain3box", 2), ("chain3box", 3)])
 @pytest.mark.parametrize("fmad", [0, 1])
 def test_virtual_ranks_bitexact(cuda_device, cfg, ranks, fmad):
     import torch
@@ -65,7 +65,8 @@ def test_virtual_ranks_bitexact(cuda_device, cfg, ranks, fmad):
     nzl = 12
     mk = {"C2": lambda nz: P.c2(nx=40, ny=24, nz=nz), "C5": lambda nz: P.c5(nx=32, ny=16, nz=nz),
           "C3": lambda nz: P.c3(nx=48, ny=20, nz=nz), "C4": c4_small,
-          "chain3": lambda nz: P.resize(P.chain3(), 20, 12, nz), "C2box": c2_boxed}[cfg]
+          "chain3": lambda nz: P.resize(P.chain3(), 20, 12, nz), "C2box": c2_boxed,
+          "chain3box": chain3_boxed}[cfg]
     glob = mk(nzl * ranks)
     plan = glob["plans"]["fused"]
     opts = {"fmad": fmad}
@@ -111,7 +112,8 @@ def test_virtual_ranks_bitexact(cuda_device, cfg, ranks, fmad):
 @pytest.mark.parametrize("cfg,ranks,mode", [("C2", 2, "fused"), ("C5", 3, "fused"), ("C3", 2, "fused"),
                                             ("C4", 2, "fused"), ("C4", 3, "unfused"),
                                             ("chain3", 3, "fused"), ("C2box", 2, "fused"),
-                                            ("C2", 3, "unfused"), ("C4", 4, "fused")])
+                                            ("C2", 3, "unfused"), ("C4", 4, "fused"),
+                                            ("chain3box", 3, "fused")])
 def test_loopback_ranks_run_bitexact(cuda_device, cfg, ranks, mode):
     """The executor's own multi-rank path (run_fused / run_unfused with a communicator:
     exchange schedule, interior planes overlapped with the exchange on the comm stream,
@@ -124,7 +126,8 @@ def test_loopback_ranks_run_bitexact(cuda_device, cfg, ranks, mode):
     nzl = 12
     mk = {"C2": lambda nz: P.c2(nx=40, ny=24, nz=nz), "C5": lambda nz: P.c5(nx=32, ny=16, nz=nz),
           "C3": lambda nz: P.c3(nx=48, ny=20, nz=nz), "C4": c4_small,
-          "chain3": lambda nz: P.resize(P.chain3(), 20, 12, nz), "C2box": c2_boxed}[cfg]
+          "chain3": lambda nz: P.resize(P.chain3(), 20, 12, nz), "C2box": c2_boxed,
+          "chain3box": chain3_boxed}[cfg]
     glob = mk(nzl * ranks)
     plan = glob["plans"]["fused"]
     dev = cuda_device
@@ -174,9 +177,21 @@ def test_loopback_ranks_run_bitexact(cuda_device, cfg, ranks, mode):
         assert torch.equal(got, want), f"{cfg} {n}: loopback multi-rank result differs from single domain"
 
 
+def chain3_boxed(nz):
+    """chain3 whose K2 (T2, read by K3 one plane above) has loop bounds crossing the slab
+    boundaries (global z in [8, 20) of 2-3 x 12 planes, x/y boxes inside the interior): in
+    the fused group the boxed stage runs one plane ahead (lead 1), so at a slab's top it is
+    evaluated on the neighbour's first plane, where outside its box it loads T2's previous
+    value — the exchange schedule must deliver T2's ghost planes (reading R2')."""
+    prog = P.resize(P.chain3(), 20, 12, nz)
+    prog["kernels"][1]["box"] = [2, 17, 1, 10, 8, 20]
+    return prog
+
+
 MK = {"C2": lambda nz: P.c2(nx=40, ny=24, nz=nz), "C5": lambda nz: P.c5(nx=32, ny=16, nz=nz),
       "C3": lambda nz: P.c3(nx=48, ny=20, nz=nz), "C4": c4_small,
-      "chain3": lambda nz: P.resize(P.chain3(), 20, 12, nz), "C2box": c2_boxed}
+      "chain3": lambda nz: P.resize(P.chain3(), 20, 12, nz), "C2box": c2_boxed,
+      "chain3box": chain3_boxed}
 
 
 @pytest.mark.parametrize("cfg,ranks,mode", [("C3", 2, "fused"), ("C3", 3, "unfused"), ("C4", 2, "fused"),

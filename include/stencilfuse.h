@@ -234,6 +234,12 @@ sp_status stencil_program_bind(stencil_program *prog, int32_t array, void *dev_p
  *   "fastpath"  1: a second, predicate-free copy of the step body for interior
  *               tiles/planes (fewer issued instructions, larger code); default 0
  *   "minblocks" __launch_bounds__ minimum resident CTAs (ptxas register budget)
+ *   "cluster_x" 2..8: fused launches with a shared-memory stage extended in x run as
+ *               thread-block clusters of that many x-neighbouring tiles; the x-halo
+ *               columns a stage needs inside a neighbour's tile are read from that
+ *               CTA's ring through distributed shared memory (remote mbarrier arrive
+ *               + ld.shared::cluster) instead of recomputed (NEXT #2); launches whose
+ *               tile columns do not divide by it stay unclustered; default 1 (off)
  *   "suspend_hint", "coef_const", "acc_split"   measured-off experiments
  *   "num_sms"   SM count assumed by the tile chooser (default 148)
  *   "l2_flush"  unused by the library (reserved) */

@@ -184,6 +184,26 @@ std::string generate_launch(const stencil_program *p, Launch &L, int index, bool
     const int NPU = (int)L.pushes.size();
     L.param_size = (L.xp_off + (L.xp ? 40 + 16 * (size_t)std::max(NPU, 1) : 0) + 63) / 64 * 64;
     const int NB = L.nbar_full, NE = L.nbar_empty;
+    // thread-block clusters along x (option cluster_x): x-halo values of shared-memory
+    // stages inside the neighbouring tile are read from that CTA's ring over DSMEM
+    // instead of recomputed; needs whole clusters (ntx % CX == 0), the TMA loader and
+    // a shared-memory stage with an x-extension
+    {
+        int cx = std::max(1, std::min(8, p->opt.cluster_x));
+        bool any_x = false;
+        for (const Stage &G : L.st)
+            if (G.needed && G.keep == Keep::Smem && (G.ex0 > 0 || G.ex1 > 0)) any_x = true;
+        if (cx > 1 && (!tma || L.xp || !any_x || L.ntx % cx != 0)) cx = 1;
+        L.cx = cx;
+    }
+    const int CX = L.cx;
+    std::vector<int> ready_of(L.st.size(), -1);  // ready mbarrier of a shared x-halo stage
+    int n_ready = 0;
+    if (CX > 1)
+        for (size_t m = 0; m < L.st.size(); ++m) {
+            const Stage &G = L.st[m];
+            if (G.needed && G.keep == Keep::Smem && (G.ex0 > 0 || G.ex1 > 0)) ready_of[m] = n_ready++;
+        }
 
     o << "// generated by stencilfuse codegen: " << (fused ? "fused group " : "original kernel ")
       << L.name << "\n#define SF_SUSPEND_HINT " << p->opt.suspend_hint
@@ -192,6 +212,7 @@ std::string generate_launch(const stencil_program *p, Launch &L, int index, bool
     o << "typedef " << T << " T;\ntypedef " << T2 << " T2;\n";
     o << "constexpr int TX = " << L.tx << ", TY = " << L.ty << ", NT = " << L.nt << ", ZC = " << L.zc
       << ", KF = " << L.kfirst << ", PF = " << L.pf << ";\n";
+    o << "constexpr int CX = " << CX << ";  // CTAs per cluster along x (DSMEM x-halo sharing)\n";
     o << "constexpr int XT = " << XT << ", YT = " << YT << ", VX = " << VX << ", VY = " << VY
       << ", CBY = " << CBY << ";  // thread (xt,yt) owns CBY blocks of VX x VY core points\n";
     o << "constexpr int NX = " << g.nx << ", NY = " << g.ny << ", NZ = " << g.nz_local
@@ -240,6 +261,9 @@ std::string generate_launch(const stencil_program *p, Launch &L, int index, bool
     o << "  const int zc = min(ZC, (lo ? p.z_mid : p.z_end) - Z0);\n";
     o << "  sf_u64 *full = (sf_u64 *)(sf_smem + " << L.bar_off << ");\n";
     if (tma) o << "  sf_u64 *empty = full + " << NB << ";\n";
+    if (CX > 1)
+        o << "  const unsigned crank = sf_cluster_rank();\n  sf_u64 *const cready = (sf_u64 *)(sf_smem + "
+          << L.ready_off << ");\n";
     for (int a = 0; a < nin; ++a) {
         const Input &I = L.in[a];
         o << "  T *const in" << a << " = (T *)(sf_smem + " << L.in_off[a] << ");  // "
@@ -309,10 +333,14 @@ std::string generate_launch(const stencil_program *p, Launch &L, int index, bool
         o << "    for (int b = 0; b < " << NB << "; ++b) sf_mbar_init(&full[b], 1);\n";
         o << "    for (int b = 0; b < " << NE << "; ++b) sf_mbar_init(&empty[b], " << L.nt / 32
           << ");\n";
+        if (n_ready)  // arrivals: every thread of each cluster neighbour, once per plane
+            o << "    for (int b = 0; b < " << n_ready << "; ++b) sf_mbar_init(&cready[b], NT * ((crank > 0) + (crank < CX - 1)));\n";
         o << "    sf_fence_mbar_init();\n";
         for (int a = 0; a < nin; ++a) o << "    sf_prefetch_tmap(&p.tm[" << a << "]);\n";
     }
     o << "  }\n  __syncthreads();\n";
+    if (CX > 1)  // the neighbours' barriers are initialised before any remote arrival
+        o << "  sf_cluster_sync();\n";
     if (L.xp) {
         // peer-push protocol: this kernel is number seq of
         // the rank's launches; a chunk within xp_dw planes of the bottom (top) slab end
@@ -365,7 +393,9 @@ std::string generate_launch(const stencil_program *p, Launch &L, int index, bool
         o << "        if (s >= KF) sf_mbar_wait(&empty[(s - KF) & " << NE - 1 << "], ((s - KF) >> "
           << log2i(NE) << ") & 1);\n";
         batch(o, "        ");
-        o << "      }\n    }\n    return;\n  }\n";
+        o << "      }\n    }\n";
+        if (CX > 1) o << "    sf_cluster_sync();  // no CTA leaves while a neighbour may read its rings\n";
+        o << "    return;\n  }\n";
     }
     // compute warps store arrays the previous group may still read (WAR) and read
     // what it wrote: wait for its completion before any global access
@@ -444,7 +474,10 @@ std::string generate_launch(const stencil_program *p, Launch &L, int index, bool
           << " : TX + x - " << left << "; }\n";
         o << "    const int gx = X0 + x, gy = Y0 + y, ax = gx + OXA, ay = gy + OYA;\n";
         o << "    h" << c << "_f[i] = ((gx >= 0 && gx < NX && gy >= 0 && gy < NY) ? 2 : 0)"
-          << " | ((ax >= 0 && ax < XP && ay >= 0 && ay < YA) ? 8 : 0);\n";
+          << " | ((ax >= 0 && ax < XP && ay >= 0 && ay < YA) ? 8 : 0)";
+        if (CX > 1)  // inside the left (16) / right (32) cluster neighbour's tile
+            o << " | ((x < 0 && crank > 0) ? 16 : 0) | ((x >= TX && crank < CX - 1) ? 32 : 0)";
+        o << ";\n";
         o << "    h" << c << "_g[i] = ay * XP + ax;\n";
         if (box_cls.count((int)c)) o << "    h" << c << "_x[i] = gx; h" << c << "_y[i] = gy;\n";
         for (const Lay &l : hlays[c])
@@ -498,6 +531,7 @@ std::string generate_launch(const stencil_program *p, Launch &L, int index, bool
     }
 
     // ------------------------------------------------------------- z-march
+    for (int r = 0; r < n_ready; ++r) o << "  unsigned cph" << r << " = 0;\n";
     o << "  for (int k = KF; k < zc; ++k) {\n";
     if (tma) {
         o << "    sf_mbar_wait(&full[(k - KF) & " << NB - 1 << "], ((k - KF) >> " << log2i(NB)
@@ -925,6 +959,7 @@ std::string generate_launch(const stencil_program *p, Launch &L, int index, bool
             };
             o << "        #pragma unroll\n        for (int i = 0; i < " << hp[c] << "; ++i) {\n";
             o << "          const int f = h" << c << "_f[i];\n";
+            if (CX > 1) o << "          if (f & 48) continue;  // the cluster neighbour computes it\n";
             // ghost points (e.g. the y-halo rows of full-height tiles) are only loaded
             o << "          T v;\n";
             if (boxed)
@@ -940,6 +975,27 @@ std::string generate_launch(const stencil_program *p, Launch &L, int index, bool
                   << "[i]] = v;\n";
             } else {
                 o << "          rh" << m << "[i][" << G.depth - 1 << "] = v;\n";
+            }
+            o << "        }\n";
+        }
+        if (ready_of[m] >= 0) {
+            // this plane of the stage is complete in this CTA: tell the cluster neighbours,
+            // wait for theirs, then copy the x-halo columns inside their tiles (same ring
+            // layout everywhere: the element TX to the left / right in the neighbour)
+            const int r = ready_of[m];
+            Lay self{true, m};
+            const std::string S = bname(self, G.lead);
+            o << "        {  // DSMEM x-halo exchange of this stage's plane\n";
+            o << "          if (crank > 0) sf_mbar_arrive_remote(sf_mapa(&cready[" << r << "], crank - 1));\n";
+            o << "          if (crank < CX - 1) sf_mbar_arrive_remote(sf_mapa(&cready[" << r << "], crank + 1));\n";
+            o << "          sf_mbar_wait_cluster(&cready[" << r << "], cph" << r << ");\n";
+            o << "          cph" << r << " ^= 1u;\n";
+            if (nh[c]) {
+                o << "          #pragma unroll\n          for (int i = 0; i < " << hp[c] << "; ++i) {\n";
+                o << "            const int f = h" << c << "_f[i], e = h" << c << "_" << lname(self) << "[i];\n";
+                o << "            if (f & 16) " << S << "[e] = sf_ld_dsmem(sf_mapa(" << S << " + e + TX, crank - 1), T(0));\n";
+                o << "            else if (f & 32) " << S << "[e] = sf_ld_dsmem(sf_mapa(" << S << " + e - TX, crank + 1), T(0));\n";
+                o << "          }\n";
             }
             o << "        }\n";
         }
@@ -990,6 +1046,7 @@ std::string generate_launch(const stencil_program *p, Launch &L, int index, bool
         o << "  if (tid == 0) sf_xs_signal(p.xs_ctr, gridDim.x * gridDim.y * gridDim.z, p.xs_self, "
              "p.xs_dn, p.xs_up, xs_seq);\n";
     }
+    if (CX > 1) o << "  sf_cluster_sync();\n";
     o << "}\n";
     L.source = o.str();
     std::ostringstream tbl;

@@ -150,6 +150,52 @@ __device__ __forceinline__ float sf_ld(const float *p) {
     return v;
 }
 
+// ---- thread-block clusters: x-halo sharing through distributed shared memory ----
+// (option cluster_x; the cluster's CTAs are x-neighbouring tiles: a stage value a
+// CTA needs inside its neighbour's tile is read from the neighbour's shared-memory
+// ring instead of being recomputed, P:L292's reason to recompute — shared memory
+// scoped to one thread block — no longer holds on sm_100a)
+__device__ __forceinline__ sf_u32 sf_cluster_rank() {
+    sf_u32 r;
+    asm volatile("mov.u32 %0, %%cluster_ctarank;" : "=r"(r));
+    return r;
+}
+// every thread of every CTA of the cluster (exited threads excluded)
+__device__ __forceinline__ void sf_cluster_sync() {
+    asm volatile("barrier.cluster.arrive.aligned;\n\tbarrier.cluster.wait.aligned;" ::: "memory");
+}
+// the address of the same shared-memory location in CTA `rank` of the cluster
+__device__ __forceinline__ sf_u32 sf_mapa(const void *p, sf_u32 rank) {
+    sf_u32 r;
+    asm volatile("mapa.shared::cluster.u32 %0, %1, %2;" : "=r"(r) : "r"(sf_smem_addr(p)), "r"(rank));
+    return r;
+}
+// arrive on an mbarrier of another CTA of the cluster; release: this thread's prior
+// shared-memory writes are visible to the waiter's acquire
+__device__ __forceinline__ void sf_mbar_arrive_remote(sf_u32 cluster_addr) {
+    asm volatile("mbarrier.arrive.release.cluster.shared::cluster.b64 _, [%0];" ::"r"(cluster_addr)
+                 : "memory");
+}
+__device__ __forceinline__ void sf_mbar_wait_cluster(sf_u64 *bar, sf_u32 parity) {
+    asm volatile(
+        "{\n\t.reg .pred P1;\n"
+        "SF_CWAIT_%=:\n\t"
+        "mbarrier.try_wait.parity.acquire.cluster.shared::cta.b64 P1, [%0], %1;\n\t"
+        "@!P1 bra SF_CWAIT_%=;\n}" ::"r"(sf_smem_addr(bar)),
+        "r"(parity)
+        : "memory");
+}
+__device__ __forceinline__ double sf_ld_dsmem(sf_u32 cluster_addr, double) {
+    double v;
+    asm volatile("ld.shared::cluster.f64 %0, [%1];" : "=d"(v) : "r"(cluster_addr) : "memory");
+    return v;
+}
+__device__ __forceinline__ float sf_ld_dsmem(sf_u32 cluster_addr, float) {
+    float v;
+    asm volatile("ld.shared::cluster.f32 %0, [%1];" : "=f"(v) : "r"(cluster_addr) : "memory");
+    return v;
+}
+
 // ---- peer-push halo protocol (several ranks, option xpush) --------------------
 // Signal block of a rank (64 B, device memory of that rank, mapped by its
 // neighbours): u64 [0] progress published by the lower neighbour, [1] by the

@@ -382,13 +382,24 @@ void launch(stencil_program *p, Mode &m, int i, void *stream, int z0, int z1, in
     int32_t ints[6] = {n_lo, z1, z2, z0, z3, 0};
     std::memcpy(base + L.int_off, ints, 24);
     void *args[] = {base};
-    if (L.pdl && !p->no_pdl) {
+    const bool use_pdl = L.pdl && !p->no_pdl;
+    if (use_pdl || L.cx > 1) {
         // programmatic dependent launch: the kernel's prologue may overlap the previous
-        // launch on the stream; griddepcontrol.wait in the kernel orders its data accesses
-        CUlaunchAttribute attr[1];
+        // launch on the stream; griddepcontrol.wait in the kernel orders its data accesses.
+        // Clusters (option cluster_x): L.cx CTAs along x per cluster
+        CUlaunchAttribute attr[2];
         std::memset(attr, 0, sizeof attr);
-        attr[0].id = CU_LAUNCH_ATTRIBUTE_PROGRAMMATIC_STREAM_SERIALIZATION;
-        attr[0].value.programmaticStreamSerializationAllowed = 1;
+        int na = 0;
+        if (use_pdl) {
+            attr[na].id = CU_LAUNCH_ATTRIBUTE_PROGRAMMATIC_STREAM_SERIALIZATION;
+            attr[na++].value.programmaticStreamSerializationAllowed = 1;
+        }
+        if (L.cx > 1) {
+            attr[na].id = CU_LAUNCH_ATTRIBUTE_CLUSTER_DIMENSION;
+            attr[na].value.clusterDim.x = (unsigned)L.cx;
+            attr[na].value.clusterDim.y = 1;
+            attr[na++].value.clusterDim.z = 1;
+        }
         CUlaunchConfig cfg;
         std::memset(&cfg, 0, sizeof cfg);
         cfg.gridDimX = (unsigned)L.ntx;
@@ -399,7 +410,7 @@ void launch(stencil_program *p, Mode &m, int i, void *stream, int z0, int z1, in
         cfg.sharedMemBytes = (unsigned)L.smem;
         cfg.hStream = (CUstream)stream;
         cfg.attrs = attr;
-        cfg.numAttrs = 1;
+        cfg.numAttrs = (unsigned)na;
         drv_check(g_drv.LaunchKernelEx(&cfg, (CUfunction)L.func, args, nullptr), "cuLaunchKernelEx");
         return;
     }

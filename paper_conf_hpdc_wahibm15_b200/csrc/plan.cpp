@@ -282,6 +282,8 @@ static void layout_launch(const stencil_program *p, Launch &L) {
     off = rup(off, 8);
     L.bar_off = off;
     off += 8 * (int64_t)L.n_bars;
+    L.ready_off = off;  // cluster plane-ready barriers (option cluster_x), one per smem stage
+    for (const Stage &G : L.st) off += G.keep == Keep::Smem ? 8 : 0;
     L.smem = rup(off, 128);
 }
 

@@ -51,6 +51,7 @@ struct Options {
                        // (r2: 40 % fewer issued instructions per step, but the doubled code
                        // overflows the 32 KB instruction cache: C4 +2 %, C2 +12 % slower)
     int minblocks = 1; // __launch_bounds__ minimum resident CTAs (register budget for ptxas)
+    int cluster_x = 1; // > 1: CTAs per cluster along x sharing x-halos of smem stages over DSMEM
     int regcap = 1; // recompile a few registers tighter when that adds a resident CTA:
                     // 0 never, 1 peer-push kernels, 2 every kernel
 };
@@ -117,6 +118,8 @@ struct Launch {
     std::vector<int> st_w, st_h, st_depth;
     int64_t bar_off = 0;
     int n_bars = 0;
+    int64_t ready_off = 0;       // cluster "plane ready" mbarriers (one per shared-memory stage)
+    int cx = 1;                  // CTAs per cluster along x (1: no cluster)
     int nbar_full = 1, nbar_empty = 1;  // per-step batch barriers (powers of two)
     // report
     double bytes_alg = 0, flops_alg = 0, bytes_exec = 0, flops_exec = 0, smem_pt = 0;

@@ -307,3 +307,29 @@ def test_ga_plan_parity_bitexact(cuda_device, cfg):
     ref = oracle_outputs(prog, seed=9)
     got = gpu_run(prog, "fused", 9, options={"fmad": 0}, plan=plan)
     assert_close(prog, got, ref, exact=True)
+
+
+CLUSTER_CASES = [("C2", lambda: P.c2(nx=96, ny=24, nz=13), ["fused"]),
+                 ("C3", lambda: P.c3(nx=128, ny=20, nz=11), ["fission_fused", "fused", "single"]),
+                 ("C5", lambda: P.c5(nx=64, ny=17, nz=9), ["fused"]),
+                 ("chain3", lambda: P.resize(P.chain3(), 70, 13, 9), ["fused"])]
+
+
+@pytest.mark.parametrize("cx", [2, 4])
+@pytest.mark.parametrize("name,mk,plans", CLUSTER_CASES, ids=[c[0] for c in CLUSTER_CASES])
+def test_cluster_dsmem_halo_bitexact(cuda_device, name, mk, plans, cx):
+    """Option cluster_x (NEXT #2): clusters of cx CTAs along x share the x-halo columns of
+    shared-memory stages through DSMEM (remote mbarrier arrive + ld.shared::cluster) instead
+    of recomputing them; fused == oracle bit-exact in the parity build, for tiles of 16
+    and 32 columns (cluster edges inside and at the global x boundary), ragged grids."""
+    from _harness import gpu_program
+    prog = mk()
+    ref = oracle_outputs(prog, seed=12)
+    clustered = 0
+    for tiles in ({}, dict(tile_x=16, tile_y=4, threads=64, block_x=1, block_y=1, block_cby=1, zchunk=4)):
+        for plan in plans:
+            p = gpu_program(prog, dict(tiles, fmad=0, cluster_x=cx), prog["plans"][plan])
+            clustered += sum("constexpr int CX = %d;" % cx in l for l in p.source("fused").splitlines())
+            got = gpu_run(prog, "fused", 12, program=p)
+            assert_close(prog, got, ref, exact=True)
+    assert clustered or cx == 4  # (a launch clusters only when its tile columns divide by cx)

@@ -153,6 +153,7 @@ std::string generate_launch(const stencil_program *p, Launch &L, int index, bool
     const bool tma = p->opt.loader == 0;
     std::ostringstream o;
     L.fn = std::string(fused ? "sf_fused_" : "sf_unfused_") + num(index);
+    L.nvtx = L.fn + " " + L.name;
     L.nth = L.nt + (tma ? 32 : 0);
     int XT, YT;
     core_geometry(L, &XT, &YT);

@@ -15,6 +15,7 @@
 #include <cuda.h>
 #include <cuda_runtime.h>
 #include <nccl.h>
+#include <nvtx3/nvToolsExt.h>
 
 #include <algorithm>
 #include <chrono>
@@ -193,6 +194,8 @@ static void exchange_loopback(stencil_program *p, const std::vector<Mode::Xfer> 
 void exchange(stencil_program *p, const std::vector<Mode::Xfer> &x, void *stream) {
     sp_comm *c = p->comm;
     if (!c || c->nranks == 1 || x.empty()) return;
+    nvtxRangePushA("stencilfuse exchange_halos");
+    struct Pop { ~Pop() { nvtxRangePop(); } } pop_range;
     for (const Mode::Xfer &t : x)
         if (!p->ptrs[t.arr]) fail(SP_E_STATE, "array '" + p->arrays[t.arr].name + "' is not bound");
     if (c->hub) {

@@ -10,6 +10,7 @@
 #include <cuda.h>
 #include <cuda_runtime.h>
 #include <nvrtc.h>
+#include <nvtx3/nvToolsExt.h>
 
 #include <atomic>
 #include <cstdio>
@@ -378,6 +379,10 @@ void launch(stencil_program *p, Mode &m, int i, void *stream, int z0, int z1, in
     const int nchunks = n_lo + n_hi;
     if (nchunks <= 0) return;
     build_params(p, m);
+    // NVTX range per group launch (SURVEY.md §5 tracing): a tool (Nsight Systems) projects
+    // it onto the kernel; a no-op without one attached
+    nvtxRangePushA(L.nvtx.c_str());
+    struct Pop { ~Pop() { nvtxRangePop(); } } pop_range;
     unsigned char *base = m.params[i][0].b;
     int32_t ints[6] = {n_lo, z1, z2, z0, z3, 0};
     std::memcpy(base + L.int_off, ints, 24);

@@ -125,6 +125,7 @@ struct Launch {
     double bytes_alg = 0, flops_alg = 0, bytes_exec = 0, flops_exec = 0, smem_pt = 0;
     // jit
     std::string fn;
+    std::string nvtx;            // NVTX range name of a launch: "<fn> <group name>"
     std::string source;
     std::string cubin;
     int regs = -1;

@@ -129,6 +129,63 @@ def check_run(rank, world, dev, cfg, mode, xpush=False, nzl=12, steps=2, grid=No
     return msg
 
 
+def check_c5_full(rank, world, dev, steps=1, n=1024, nz_total=1024):
+    """BASELINE configs[4] at full size: C5 (3 tracers x gradient/flux/divergence/update,
+    12 kernels) on 1024 x 1024 x 128 planes per GPU, 1024^3 fp64 in total at 8 ranks,
+    fused plan, real NCCL halo exchange overlapped with the interior planes.  P9 at full
+    scale: rank 0 also runs the undecomposed 1024^3 grid on its GPU (~138 GB of HBM) and
+    compares SHA-1 digests of every rank's OUT slab with the same planes of the single
+    domain (bit for bit)."""
+    import hashlib
+    import torch
+    import torch.distributed as dist
+    import bench
+    from paper_conf_hpdc_wahibm15_b200 import Comm, Program
+    from synth import programs as P
+    nzl = nz_total // world
+    loc = P.c5(nx=n, ny=n, nz=nzl)
+    plan = loc["plans"]["fused"]
+    probe = Program(loc, nz_global=nzl * world)
+    probe.set_plan(plan)
+    zhalo = max([max(r["z_below"], r["z_above"]) for r in probe.reports("fused")] + [1])
+    del probe
+    comm = Comm(rank, world)
+    s = Program(loc, comm=comm, nz_global=nzl * world, z_offset=rank * nzl, zhalo=zhalo)
+    s.set_plan(plan)
+    s.allocate(dev, fill=0.0)
+    bench.fill_inputs(s, loc, dev, rank * nzl, zhalo)
+    s.load("fused")
+    torch.cuda.synchronize(dev)
+    dist.barrier()
+    for _ in range(steps):
+        s.run_fused()
+    torch.cuda.synchronize(dev)
+    outs = [a["name"] for a in loc["arrays"] if a["role"] in ("out", "inout")]
+    mine = {nm: hashlib.sha1(s.interior_view(s.tensors[nm]).cpu().numpy().tobytes()).hexdigest()
+            for nm in outs}
+    del s, comm
+    torch.cuda.empty_cache()
+    got = [None] * world if rank == 0 else None
+    dist.gather_object(mine, got, dst=0)
+    if rank == 0:
+        glob = P.c5(nx=n, ny=n, nz=nzl * world)
+        single = Program(glob)
+        single.set_plan(plan)
+        single.allocate(dev, fill=0.0)
+        bench.fill_inputs(single, glob, dev, 0, glob["grid"]["ghost"][2])
+        for _ in range(steps):
+            single.run_fused()
+        torch.cuda.synchronize(dev)
+        for nm in outs:
+            full = single.interior_view(single.tensors[nm])
+            for r in range(world):
+                want = hashlib.sha1(full[r * nzl:(r + 1) * nzl].cpu().numpy().tobytes()).hexdigest()
+                assert got[r][nm] == want, f"C5 {n}^2x{nz_total} x{world}: {nm} slab {r} differs"
+        del single
+    dist.barrier()
+    return f"C5 {n}^2x{nz_total} fused x{world}: bit-exact with the single domain (SHA-1 per slab)"
+
+
 CASES = [("C2", "fused", False), ("C2", "unfused", False), ("C4", "fused", False),
          ("C4", "unfused", False), ("C5", "fused", False), ("C3", "fused", False),
          ("C4", "fused", True)]
@@ -154,6 +211,10 @@ def worker(rank, world, device_index, cases=None, q=None, port=None, env=None):
         out.append(check_exchange_halos(rank, world, dev))
         for cfg, mode, xpush in (CASES if cases is None else cases):
             out.append(check_run(rank, world, dev, cfg, mode, xpush))
+        if os.environ.get("SF_MULTIGPU_C5_FULL") == "1" and world == 8:
+            out.append(check_c5_full(rank, world, dev))
+        elif os.environ.get("SF_MULTIGPU_C5_FULL") == "small":  # the same check, reduced
+            out.append(check_c5_full(rank, world, dev, n=96, nz_total=48 * world))
         if q is not None:
             q.put((rank, "ok", out))
     except Exception:

@@ -34,7 +34,8 @@ def _run_two_ranks(cases, timeout=900):
     ctx = mp.get_context("spawn")
     q = ctx.Queue()
     port = _free_port()
-    ps = [ctx.Process(target=worker, args=(r, 2, 0, cases, q, port, single_gpu_nccl_env(r)))
+    ps = [ctx.Process(target=worker, args=(r, 2, 0, cases, q, port,
+                                           dict(single_gpu_nccl_env(r), SF_MULTIGPU_C5_FULL="small")))
           for r in range(2)]
     for p in ps:
         p.start()
@@ -57,7 +58,7 @@ def test_nccl_exchange_halos_and_runs_two_processes(cuda_device):
     from _nccl_worker import CASES
     out = _run_two_ranks(CASES)
     print("\n".join(out))
-    assert len(out) == 1 + len(CASES)
+    assert len(out) == 2 + len(CASES)
 
 
 def test_bench_multirank_path_two_processes(cuda_device):

@@ -570,3 +570,20 @@ def test_lazy_fission_search_model_objective():
             assert rep["fissioned_kernels"] == 1
             k0 = [g for g in plan if any(r.startswith("K0:") for r in g)]
             assert len(k0) == 2 and any(len(g) > 1 for g in k0)
+
+
+def test_bench_refuses_gpu_count_mismatch():
+    """bench.py never reports an N-GPU run that is not one: --gpus != WORLD_SIZE
+    under torchrun, or --gpus N > visible devices without it, exits non-zero before any work."""
+    import subprocess
+    import sys
+    bench = os.path.join(ROOT, "bench.py")
+    env = dict(os.environ, WORLD_SIZE="2", RANK="0", LOCAL_RANK="0")
+    r = subprocess.run([sys.executable, bench, "--gpus", "4"], capture_output=True, text=True, env=env,
+                       timeout=120)
+    assert r.returncode != 0 and "WORLD_SIZE=2" in r.stderr
+    env = {k: v for k, v in os.environ.items() if k not in ("WORLD_SIZE", "RANK", "LOCAL_RANK")}
+    env["CUDA_VISIBLE_DEVICES"] = ""
+    r = subprocess.run([sys.executable, bench, "--gpus", "2"], capture_output=True, text=True, env=env,
+                       timeout=300)
+    assert r.returncode != 0 and "CUDA device" in r.stderr

@@ -24,8 +24,11 @@ def _ngpus():
     return torch.cuda.device_count()
 
 
-@pytest.mark.parametrize("n", [2, 4, 8])
-def test_torchrun_nccl_ranks(n):
+@pytest.mark.parametrize("n,c5_full", [(2, False), (4, False), (8, False), (8, True)],
+                         ids=["2", "4", "8", "8-C5-1024cubed"])
+def test_torchrun_nccl_ranks(n, c5_full):
+    """c5_full: additionally BASELINE configs[4] at full size (1024^3 fp64 over 8 GPUs),
+    bit-exact against the undecomposed grid run on GPU 0 (tests/_nccl_worker.check_c5_full)."""
     have = _ngpus()
     if have < n:
         pytest.skip(f"needs {n} GPUs, {have} visible")
@@ -36,6 +39,7 @@ def test_torchrun_nccl_ranks(n):
     cmd = [sys.executable, "-m", "torch.distributed.run", "--nnodes=1", f"--nproc-per-node={n}",
            "--master-addr=127.0.0.1", f"--master-port={port}",
            os.path.join(ROOT, "tests", "_nccl_worker.py")]
-    r = subprocess.run(cmd, capture_output=True, text=True, timeout=1800)
+    env = dict(os.environ, SF_MULTIGPU_C5_FULL="1" if c5_full else "0")
+    r = subprocess.run(cmd, capture_output=True, text=True, timeout=3600, env=env)
     print(r.stdout[-4000:])
     assert r.returncode == 0 and "MULTIGPU_OK" in r.stdout, r.stderr[-4000:]

@@ -469,3 +469,22 @@ def test_openmp_build_identical(cfg):
     OracleProgram(prog, parallel=True).run(b)
     for k in a:
         assert a[k].tobytes() == b[k].tobytes(), k
+
+
+def test_wide_variant_pinned_to_independent_binary64_evaluator():
+    """oracle_run_f32_in_f64 (binary64 arithmetic on binary32 storage, used as the fp32
+    error-bound reference) equals the independent NumPy slicing evaluator run in binary64
+    (double coefficients, fp32 arrays promoted, each statement's result rounded to fp32
+    when stored) bit for bit, on random fp32 programs with products and loop bounds."""
+    import _numpy_eval
+    from _fuzz import random_lib_program
+    for seed in range(10):
+        rng = np.random.default_rng(700 + seed)
+        prog = random_lib_program(rng, n=(7, 5, 4), dtype="f32", boxes=seed % 2 == 1)
+        a = dense_arrays(prog, seed=seed)
+        w = {k: v.copy() for k, v in a.items()}
+        OracleProgram(prog).run(w, wide=True)
+        ref = _numpy_eval.run(dict(prog, dtype="f64"), {k: v.copy() for k, v in a.items()})
+        for name in w:
+            assert w[name].dtype == np.float32
+            assert w[name].tobytes() == ref[name].astype(np.float32).tobytes(), (seed, name)

@@ -316,7 +316,9 @@ typedef struct {
  * each one that fits and costs its fastest; `configs` (nullable, >= cap entries,
  * written with the groups) receives each returned group's configuration for
  * sp_plan_tune (all zero: the chooser's).  Output as sp_plan_greedy; `report`
- * (nullable) receives costs and counts. */
+ * (nullable) receives costs and counts.  Does not set the plan.  Errors: SP_E_ARG
+ * (options), SP_E_STATE (measured: an array not bound), SP_E_JIT / SP_E_CUDA
+ * (measured: compilation or a kernel failed). */
 typedef struct {
     int32_t generations;        /* GA generations (0: pre-step + DP + seeds only)            */
     int32_t population;         /* GA population (clamped to >= 4)                            */

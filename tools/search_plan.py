@@ -72,6 +72,13 @@ def main():
     for g, c in zip(out["groups"], out["configs"]):
         print(g, c)
     if a.out:
+        if a.workload != "C4" and os.path.exists(a.out):
+            # C2/C3/C5 plan files hold named plans: add / replace the "searched" entry
+            pj = json.load(open(a.out))
+            pj.setdefault("plans", {})["searched"] = {"groups": out["groups"], "configs": out["configs"],
+                                                      "planner": out["planner"],
+                                                      "search_report": out["search_report"]}
+            out = pj
         json.dump(out, open(a.out, "w"), indent=1)
         print("wrote", a.out)
 

@@ -618,7 +618,7 @@ std::string generate_launch(const stencil_program *p, Launch &L, int index, bool
         if (G.needed && p->stmts[G.gid].boxed) any_boxed = true;
     const bool spec = p->opt.fastpath && !any_boxed;
     if (spec) {
-        int smin = INT32_MAX, kst0 = INT32_MIN;
+        int kst0 = INT32_MIN;
         int lmin = INT32_MAX, lmax = INT32_MIN, slmin = INT32_MAX, slmax = INT32_MIN;
         for (const Stage &G : L.st) {
             if (!G.needed) continue;
@@ -627,7 +627,6 @@ std::string generate_launch(const stencil_program *p, Launch &L, int index, bool
             lmax = std::max(lmax, G.lead);
             if (G.stored) { slmin = std::min(slmin, G.lead); slmax = std::max(slmax, G.lead); }
         }
-        (void)smin;
         o << "    // fast-step window [sf_k0, sf_k1) of this chunk (see codegen.cpp)\n";
         o << "    int sf_k0 = max(" << kst0 << ", ZLO - Z0 - (" << lmin << ")), sf_k1 = min(zc, ZHI - Z0 - ("
           << lmax << "));\n";

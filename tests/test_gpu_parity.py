@@ -333,3 +333,26 @@ def test_cluster_dsmem_halo_bitexact(cuda_device, name, mk, plans, cx):
             got = gpu_run(prog, "fused", 12, program=p)
             assert_close(prog, got, ref, exact=True)
     assert clustered or cx == 4  # (a launch clusters only when its tile columns divide by cx)
+
+
+DEGENERATE = [(1, 1, 1), (1, 7, 3), (5, 1, 1), (3, 2, 1), (2, 1, 9), (17, 1, 2)]
+
+
+@pytest.mark.parametrize("n", DEGENERATE, ids=["x".join(map(str, n)) for n in DEGENERATE])
+def test_degenerate_grids_bitexact(cuda_device, n):
+    """Degenerate interiors (a single point, single rows / columns / planes): every ghost
+    rule (R1) is in play at once, tiles are mostly outside the interior, z-chunks have one
+    plane.  Unfused, fused (incl. fission + fusion) and a kernel with an EMPTY loop box
+    (R2': writes nothing) in the parity build, bit-exact with the oracle."""
+    cases = [(P.resize(P.c2(), *n), ["fused"]), (P.resize(P.c3(), *n), ["fused", "fission_fused"]),
+             (P.resize(P.chain3(), *n), ["fused"])]
+    boxed = P.resize(P.chain3(), *n)
+    boxed["kernels"][1]["box"] = [0, 0, 0, n[1], 0, n[2]]  # empty in x: T2 keeps its stored value
+    cases.append((boxed, ["fused"]))
+    for prog, plans in cases:
+        ref = oracle_outputs(prog, seed=13, poison=False)
+        got = gpu_run(prog, "unfused", 13, options={"fmad": 0}, poison=False)
+        assert_close(prog, got, ref, exact=True)
+        for plan in plans:
+            got = gpu_run(prog, "fused", 13, options={"fmad": 0}, plan=prog["plans"][plan], poison=False)
+            assert_close(prog, got, ref, exact=True)

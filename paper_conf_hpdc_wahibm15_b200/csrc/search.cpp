@@ -166,6 +166,10 @@ class MeasuredObjective : public Objective {
         }
         if (m.launches.empty()) return;
         m.analyzed = true;
+        struct Unload {  // modules of this batch are unloaded on every exit path
+            Mode &m;
+            ~Unload() { unload_mode(m); }
+        } unload{m};
         compile_mode(p_, m);
         load_mode(p_, m);
         if (!flush_) {
@@ -203,7 +207,6 @@ class MeasuredObjective : public Objective {
                 cfg_[k] = owner[j].second;
             }
         }
-        unload_mode(m);
     }
 
   private:

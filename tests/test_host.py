@@ -587,3 +587,40 @@ def test_bench_refuses_gpu_count_mismatch():
     r = subprocess.run([sys.executable, bench, "--gpus", "2"], capture_output=True, text=True, env=env,
                        timeout=300)
     assert r.returncode != 0 and "CUDA device" in r.stderr
+
+
+def test_exchange_schedule_includes_boxed_stage_previous_value():
+    """Reading R2' on several ranks: a boxed statement evaluated on a plane beyond the slab
+    (lead 1 here: K2's T2 is read one plane above by K3) loads T2's previous value outside
+    its box there, so the schedule receives T2's ghost plane above (and nothing below),
+    besides A's step-start planes; without loop bounds T2 is never exchanged (it is
+    computed on chip everywhere)."""
+    from paper_conf_hpdc_wahibm15_b200 import Comm
+    prog = P.resize(P.chain3(), 20, 12, 12)
+    comms = Comm.loopback(2)
+    q = Program(prog, comm=comms[0], nz_global=24, z_offset=0, zhalo=2)
+    q.set_plan(prog["plans"]["fused"])
+    assert [x for x in q.exchange_plan("fused", 0) if x[0] == "T2"] == []
+    prog["kernels"][1]["box"] = [2, 17, 1, 10, 8, 20]
+    q = Program(prog, comm=comms[0], nz_global=24, z_offset=0, zhalo=2)
+    q.set_plan(prog["plans"]["fused"])
+    assert ("T2", 0, 1) in q.exchange_plan("fused", 0)
+
+
+def test_live_out_stores_writer_before_boxed_rewrite():
+    """Reading R2' / R6: when a later group rewrites X only inside a box, the earlier
+    writer of X must store it (the boxed statement loads the old value outside its box) —
+    the bug the round-2 legal-plan fuzz exposed.  Here T (a TEMP) is written by K1 and
+    rewritten in a box by K2 in the next group, then read by K3: group 0 stores T."""
+    T = P.tap
+    prog = {"name": "boxlive", "dtype": "f64", "grid": {"nx": 8, "ny": 6, "nz": 4, "ghost": [1, 1, 1]},
+            "arrays": [{"name": n, "role": r} for n, r in (("A", "in"), ("T", "temp"), ("O", "out"))],
+            "kernels": [P.kernel("K1", P.stmt("T", [{"c": 2.0, "a": T("A", (0, 0, 0))}])),
+                        dict(P.kernel("K2", P.stmt("T", [{"c": 3.0, "a": T("A", (1, 0, 0))}])),
+                             box=[1, 4, 0, 6, 0, 4]),
+                        P.kernel("K3", P.stmt("O", [{"c": 1.0, "a": T("T", (0, 0, 0))}]))]}
+    p = Program(prog)
+    p.set_plan([["K1"], ["K2", "K3"]])
+    assert p.report("fused", 0)["n_stores"] == 1
+    p.set_plan([["K1"], ["K2"], ["K3"]])
+    assert [r["n_stores"] for r in p.reports("fused")] == [1, 1, 1]

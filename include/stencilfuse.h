@@ -285,6 +285,7 @@ sp_status sp_plan_greedy(stencil_program *prog, int32_t cap, int32_t *n_groups,
 typedef struct {
     int32_t tile_x, tile_y, zchunk, threads, prefetch, block_x, block_y, block_cby;
     int32_t zqueue;
+    int32_t fastpath;  /* 0 = the program's "fastpath" option, 1 = off, 2 = on (this launch) */
 } sp_tile_config;
 
 /* Lazy-fission plan search (the paper's search step,

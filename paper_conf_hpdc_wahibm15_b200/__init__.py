@@ -379,14 +379,15 @@ class Program:
 
     def tune(self, mode, i, cfg):
         """Pin launch i's configuration: dict with tile_x, tile_y, zchunk, threads, prefetch,
-        block_x, block_y, block_cby (missing/0 = chooser) and zqueue (the option's values
-        0/1/2; missing = the program option); None removes the pin."""
+        block_x, block_y, block_cby (missing/0 = chooser), zqueue (the option's values
+        0/1/2) and fastpath (0/1; missing = the program option); None removes the pin."""
         if cfg is None:
             _check(lib().sp_plan_tune(self.handle, self._mode(mode), i, None))
             return
         vals = {k: int(v) for k, v in cfg.items() if k in dict(SpTileConfig._fields_)}
-        if "zqueue" in vals:
-            vals["zqueue"] += 1  # ABI: 0 = inherit, policy + 1 otherwise
+        for k in ("zqueue", "fastpath"):
+            if k in vals:
+                vals[k] += 1  # ABI: 0 = inherit the program option, value + 1 otherwise
         c = SpTileConfig(**vals)
         _check(lib().sp_plan_tune(self.handle, self._mode(mode), i, ctypes.byref(c)))
 

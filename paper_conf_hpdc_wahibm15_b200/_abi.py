@@ -53,7 +53,7 @@ class SpLayout(ctypes.Structure):
 
 class SpTileConfig(ctypes.Structure):
     _fields_ = [(n, ctypes.c_int32) for n in ("tile_x", "tile_y", "zchunk", "threads", "prefetch",
-                                              "block_x", "block_y", "block_cby", "zqueue")]
+                                              "block_x", "block_y", "block_cby", "zqueue", "fastpath")]
 
 
 class SpSearchOptions(ctypes.Structure):

@@ -616,7 +616,7 @@ std::string generate_launch(const stencil_program *p, Launch &L, int index, bool
     bool any_boxed = false;
     for (const Stage &G : L.st)
         if (G.needed && p->stmts[G.gid].boxed) any_boxed = true;
-    const bool spec = p->opt.fastpath && !any_boxed;
+    const bool spec = (L.fastpath >= 0 ? L.fastpath : p->opt.fastpath) && !any_boxed;
     if (spec) {
         int kst0 = INT32_MIN;
         int lmin = INT32_MAX, lmax = INT32_MIN, slmin = INT32_MAX, slmax = INT32_MIN;

@@ -566,6 +566,7 @@ void analyze_mode(stencil_program *p, bool fused, const std::vector<std::vector<
                 if (c.block_y) p->opt.block_y = c.block_y;
                 if (c.block_cby) p->opt.block_cby = c.block_cby;
                 if (c.zqueue) p->opt.zqueue = c.zqueue - 1;
+                if (c.fastpath) L.fastpath = c.fastpath - 1;
                 try {
                     choose_config(p, L);
                 } catch (...) {

@@ -84,6 +84,7 @@ class Objective {
                 if (pin->block_y) p_->opt.block_y = pin->block_y;
                 if (pin->block_cby) p_->opt.block_cby = pin->block_cby;
                 if (pin->zqueue) p_->opt.zqueue = pin->zqueue - 1;
+                if (pin->fastpath) L.fastpath = pin->fastpath - 1;
             }
             choose_config(p_, L, quick);
             p_->opt = saved;

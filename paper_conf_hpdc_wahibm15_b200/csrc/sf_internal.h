@@ -142,6 +142,7 @@ struct Launch {
     size_t xp_off = 0;       // param offset of the peer-push section
     bool dead = false;       // nothing to compute (all stages dead)
     bool pdl = false;        // launched with programmatic stream serialization
+    int fastpath = -1;       // per-launch pin of the "fastpath" codegen variant (-1: option)
 };
 
 struct Mode {

@@ -328,8 +328,13 @@ class Program:
         "measured" (groups JIT-compiled and timed on the current device at the chooser's
         and each candidate configuration in `configs`; arrays must be bound).  Returns
         (plan, report dict) or, with_configs, (plan, per-group configuration dicts, report)."""
-        cands = [SpTileConfig(**{k: int(v) for k, v in c.items() if k in dict(SpTileConfig._fields_)})
-                 for c in (configs or [])]
+        def abi(c):  # option-level dict (as for tune) -> ABI values (zqueue/fastpath + 1)
+            v = {k: int(x) for k, x in c.items() if k in dict(SpTileConfig._fields_)}
+            for k in ("zqueue", "fastpath"):
+                if k in v:
+                    v[k] += 1
+            return SpTileConfig(**v)
+        cands = [abi(c) for c in (configs or [])]
         carr = (SpTileConfig * max(1, len(cands)))(*cands)
         o = SpSearchOptions(generations=int(generations), population=int(population),
                             seed=int(seed), objective={"model": 0, "measured": 1}[objective],
@@ -351,8 +356,13 @@ class Program:
         report = {f: getattr(rep, f) for f, _ in SpSearchReport._fields_}
         if not with_configs:
             return plan, report
-        cfgs = [{f: getattr(out_cfg[g], f) for f, _ in SpTileConfig._fields_ if getattr(out_cfg[g], f)}
-                or None for g in range(ng.value)]
+        cfgs = []
+        for g in range(ng.value):
+            c = {f: getattr(out_cfg[g], f) for f, _ in SpTileConfig._fields_ if getattr(out_cfg[g], f)}
+            for k in ("zqueue", "fastpath"):  # back to option-level values (as tune() takes)
+                if k in c:
+                    c[k] -= 1
+            cfgs.append(c or None)
         return plan, cfgs, report
 
     def n_launches(self, mode):

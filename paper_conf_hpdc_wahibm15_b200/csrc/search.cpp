@@ -153,6 +153,7 @@ class MeasuredObjective : public Objective {
                 std::memset(&c, 0, sizeof c);
                 c.tile_x = L.tx; c.tile_y = L.ty; c.zchunk = L.zc; c.threads = L.nt; c.prefetch = L.pf;
                 c.block_x = L.vx; c.block_y = L.vy; c.block_cby = L.cby;
+                c.fastpath = L.fastpath >= 0 ? L.fastpath + 1 : 0;
                 bool dup = false;
                 for (const auto &o : owner)
                     dup |= o.first == i && !std::memcmp(&o.second, &c, sizeof c);

@@ -30,8 +30,14 @@ CANDIDATES = [
     dict(tile_x=32, tile_y=16, threads=128, block_x=2, block_y=2, block_cby=1, zchunk=16, prefetch=3),
     dict(tile_x=32, tile_y=8, threads=128, block_x=1, block_y=2, block_cby=1, zchunk=32, prefetch=2),
 ]
-# the predicate-free step body as a per-group variant of the shapes the C4 groups pin
-CANDIDATES += [dict(c, fastpath=1) for c in CANDIDATES[:4]]
+CANDIDATES += [
+    dict(tile_x=64, tile_y=8, threads=128, block_x=2, block_y=2, block_cby=1, zchunk=16, prefetch=2),
+    dict(tile_x=32, tile_y=16, threads=128, block_x=1, block_y=4, block_cby=1, zchunk=16, prefetch=3),
+    dict(tile_x=32, tile_y=8, threads=64, block_x=2, block_y=2, block_cby=1, zchunk=16, prefetch=2),
+    dict(tile_x=32, tile_y=8, threads=128, block_x=1, block_y=2, block_cby=1, zchunk=32, prefetch=3),
+]
+# the predicate-free step body (codegen option "fastpath") as a per-group variant of each shape
+CANDIDATES += [dict(c, fastpath=1) for c in list(CANDIDATES)]
 
 
 def measured_search(workload, generations=12, population=16, seed=1, candidates=CANDIDATES, reps=3):

@@ -36,16 +36,26 @@ CANDIDATES += [
     dict(tile_x=32, tile_y=8, threads=64, block_x=2, block_y=2, block_cby=1, zchunk=16, prefetch=2),
     dict(tile_x=32, tile_y=8, threads=128, block_x=1, block_y=2, block_cby=1, zchunk=32, prefetch=3),
 ]
+# fp32 shapes (C3): wider tiles, 4-float register blocks (LDS.128 / STG.128)
+CANDIDATES_F32 = [
+    dict(tile_x=64, tile_y=8, threads=128, block_x=4, block_y=2, block_cby=1, zchunk=16, prefetch=2),
+    dict(tile_x=128, tile_y=8, threads=128, block_x=4, block_y=4, block_cby=1, zchunk=16, prefetch=2),
+    dict(tile_x=64, tile_y=16, threads=128, block_x=2, block_y=4, block_cby=1, zchunk=16, prefetch=2),
+    dict(tile_x=128, tile_y=4, threads=128, block_x=4, block_y=1, block_cby=1, zchunk=32, prefetch=2),
+]
 # the predicate-free step body (codegen option "fastpath") as a per-group variant of each shape
 CANDIDATES += [dict(c, fastpath=1) for c in list(CANDIDATES)]
+CANDIDATES_F32 += [dict(c, fastpath=1) for c in list(CANDIDATES_F32)]
 
 
-def measured_search(workload, generations=12, population=16, seed=1, candidates=CANDIDATES, reps=3):
+def measured_search(workload, generations=12, population=16, seed=1, candidates=None, reps=3):
     """Run the search on a full-size instance of the workload; returns the plan-file dict."""
     import torch
     import bench
     from paper_conf_hpdc_wahibm15_b200 import Program
     prog = bench.load_workload(workload)
+    if candidates is None:
+        candidates = CANDIDATES + (CANDIDATES_F32 if prog["dtype"] == "f32" else [])
     dev = torch.device("cuda:0")
     p = Program(prog)
     p.allocate(dev, fill=0.0)

@@ -109,12 +109,15 @@ def test_virtual_ranks_bitexact(cuda_device, cfg, ranks, fmad):
         assert torch.equal(got, want), f"{cfg} {n}: slab result differs from single domain"
 
 
-@pytest.mark.parametrize("cfg,ranks,mode", [("C2", 2, "fused"), ("C5", 3, "fused"), ("C3", 2, "fused"),
-                                            ("C4", 2, "fused"), ("C4", 3, "unfused"),
-                                            ("chain3", 3, "fused"), ("C2box", 2, "fused"),
-                                            ("C2", 3, "unfused"), ("C4", 4, "fused"),
-                                            ("chain3box", 3, "fused")])
-def test_loopback_ranks_run_bitexact(cuda_device, cfg, ranks, mode):
+@pytest.mark.parametrize("cfg,ranks,mode,opts", [("C2", 2, "fused", {}), ("C5", 3, "fused", {}),
+                                                 ("C3", 2, "fused", {}), ("C4", 2, "fused", {}),
+                                                 ("C4", 3, "unfused", {}), ("chain3", 3, "fused", {}),
+                                                 ("C2box", 2, "fused", {}), ("C2", 3, "unfused", {}),
+                                                 ("C4", 4, "fused", {}), ("chain3box", 3, "fused", {}),
+                                                 ("C4", 3, "fused", {"fastpath": 1}),
+                                                 ("C5", 2, "fused", {"fastpath": 1}),
+                                                 ("C3", 3, "unfused", {"fastpath": 1})])
+def test_loopback_ranks_run_bitexact(cuda_device, cfg, ranks, mode, opts):
     """The executor's own multi-rank path (run_fused / run_unfused with a communicator:
     exchange schedule, interior planes overlapped with the exchange on the comm stream,
     boundary planes after its event, no PDL) on in-process virtual ranks, one host
@@ -145,7 +148,10 @@ def test_loopback_ranks_run_bitexact(cuda_device, cfg, ranks, mode):
     comms = Comm.loopback(ranks)
     slabs = []
     for r in range(ranks):
-        s = Program(loc, comm=comms[r], nz_global=nzl * ranks, z_offset=r * nzl, zhalo=zhalo)
+        # opts: codegen variants (e.g. the fastpath step body, whose fast-step window must
+        # treat deep-halo planes of the global interior like interior planes)
+        s = Program(loc, comm=comms[r], nz_global=nzl * ranks, z_offset=r * nzl, zhalo=zhalo,
+                    options=opts)
         s.set_plan(plan)
         s.allocate(dev)
         fill(s, loc, dev, r * nzl, zhalo, nz_global=nzl * ranks)

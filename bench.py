@@ -194,6 +194,10 @@ def run_ours(args):
     del probe
     comm = Comm(rank, world) if world > 1 else None
     xpush = bool(args.xpush and world > 1)
+    if xpush and os.environ.get("SF_BENCH_SHARE_GPU") == "1":
+        # peer-push kernels spin on flags the neighbour's kernels set; ranks sharing one
+        # GPU have no co-residency guarantee (Xid 109 recorded on this driver)
+        raise SystemExit("--xpush needs one GPU per rank (not with SF_BENCH_SHARE_GPU=1)")
     p = Program(prog, comm=comm, nz_global=nz * world, z_offset=rank * nz, zhalo=zhalo,
                 options={"xpush": 1} if xpush else None)
     p.set_plan(plan)

@@ -368,7 +368,9 @@ def _ipc_worker(rank, world, port, cfg, q, concurrent=False):
         dist.destroy_process_group()
 
 
-@pytest.mark.parametrize("cfg,concurrent", [("C4", False), ("C3", False), ("C4", True), ("C3", True)])
+# lockstep only: concurrent launches whose kernels wait on the other process's kernels are
+# not run on one GPU (no co-residency guarantee; Xid 109 recorded on this driver)
+@pytest.mark.parametrize("cfg,concurrent", [("C4", False), ("C3", False)])
 def test_peer_push_ipc_processes(cuda_device, cfg, concurrent):
     """Peer push across PROCESSES (the real deployment shape: one process per rank):
     each rank maps its neighbours' TEMP buffers and signal blocks with CUDA IPC

@@ -56,9 +56,14 @@ def _run_two_ranks(cases, timeout=900):
 
 def test_nccl_exchange_halos_and_runs_two_processes(cuda_device):
     from _nccl_worker import CASES
-    out = _run_two_ranks(CASES)
+    # xpush kernels of one rank spin on flags the other rank's kernels set: on ONE GPU two
+    # processes' waiting kernels are not guaranteed to be co-resident (the profiling guide
+    # records Xid 109 context-switch timeouts for exactly that), so the concurrent peer-push
+    # case runs only where each rank has its own GPU (tests/test_multigpu.py)
+    cases = [c for c in CASES if not c[2]]
+    out = _run_two_ranks(cases)
     print("\n".join(out))
-    assert len(out) == 2 + len(CASES)
+    assert len(out) == 2 + len(cases)
 
 
 def test_bench_multirank_path_two_processes(cuda_device):

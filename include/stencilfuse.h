@@ -234,6 +234,12 @@ sp_status stencil_program_bind(stencil_program *prog, int32_t array, void *dev_p
  *   "fastpath"  1: a second, predicate-free copy of the step body for interior
  *               tiles/planes (fewer issued instructions, larger code); default 0
  *   "minblocks" __launch_bounds__ minimum resident CTAs (ptxas register budget)
+ *   "frame"     1: region-vector evaluation of fused launches: every statement is
+ *               evaluated on its whole extended region (tile + halo of complex
+ *               fusion, §5.5.3) in 16-byte x-vectors of adjacent points
+ *               enumerated linearly over the threads, instead of register blocks on
+ *               the tile plus point-wise halo strips; launches with loop-bounded
+ *               statements, peer push or clusters keep the block form; default 0
  *   "cluster_x" 2..8: fused launches with a shared-memory stage extended in x run as
  *               thread-block clusters of that many x-neighbouring tiles; the x-halo
  *               columns a stage needs inside a neighbour's tile are read from that
@@ -286,6 +292,7 @@ typedef struct {
     int32_t tile_x, tile_y, zchunk, threads, prefetch, block_x, block_y, block_cby;
     int32_t zqueue;
     int32_t fastpath;  /* 0 = the program's "fastpath" option, 1 = off, 2 = on (this launch) */
+    int32_t frame;     /* 0 = the program's "frame" option, 1 = off, 2 = on (this launch) */
 } sp_tile_config;
 
 /* Lazy-fission plan search (the paper's search step,

@@ -330,7 +330,7 @@ class Program:
         (plan, report dict) or, with_configs, (plan, per-group configuration dicts, report)."""
         def abi(c):  # option-level dict (as for tune) -> ABI values (zqueue/fastpath + 1)
             v = {k: int(x) for k, x in c.items() if k in dict(SpTileConfig._fields_)}
-            for k in ("zqueue", "fastpath"):
+            for k in ("zqueue", "fastpath", "frame"):
                 if k in v:
                     v[k] += 1
             return SpTileConfig(**v)
@@ -359,7 +359,7 @@ class Program:
         cfgs = []
         for g in range(ng.value):
             c = {f: getattr(out_cfg[g], f) for f, _ in SpTileConfig._fields_ if getattr(out_cfg[g], f)}
-            for k in ("zqueue", "fastpath"):  # back to option-level values (as tune() takes)
+            for k in ("zqueue", "fastpath", "frame"):  # back to option-level values (as tune() takes)
                 if k in c:
                     c[k] -= 1
             cfgs.append(c or None)
@@ -390,12 +390,12 @@ class Program:
     def tune(self, mode, i, cfg):
         """Pin launch i's configuration: dict with tile_x, tile_y, zchunk, threads, prefetch,
         block_x, block_y, block_cby (missing/0 = chooser), zqueue (the option's values
-        0/1/2) and fastpath (0/1; missing = the program option); None removes the pin."""
+        0/1/2), fastpath and frame (0/1; missing = the program option); None removes the pin."""
         if cfg is None:
             _check(lib().sp_plan_tune(self.handle, self._mode(mode), i, None))
             return
         vals = {k: int(v) for k, v in cfg.items() if k in dict(SpTileConfig._fields_)}
-        for k in ("zqueue", "fastpath"):
+        for k in ("zqueue", "fastpath", "frame"):
             if k in vals:
                 vals[k] += 1  # ABI: 0 = inherit the program option, value + 1 otherwise
         c = SpTileConfig(**vals)

@@ -53,7 +53,8 @@ class SpLayout(ctypes.Structure):
 
 class SpTileConfig(ctypes.Structure):
     _fields_ = [(n, ctypes.c_int32) for n in ("tile_x", "tile_y", "zchunk", "threads", "prefetch",
-                                              "block_x", "block_y", "block_cby", "zqueue", "fastpath")]
+                                              "block_x", "block_y", "block_cby", "zqueue", "fastpath",
+                                              "frame")]
 
 
 class SpSearchOptions(ctypes.Structure):

@@ -102,10 +102,37 @@ static std::map<PosKey, PosInfo> block_positions(const Launch &L, const Stage &G
     return pos;
 }
 
+// Region-vector ("frame") evaluation of a statement: its region rows [y_lo, y_lo+rows)
+// and x-vector columns [x_lo, x_lo + cs*VW) relative to the tile (x rounded out to the
+// 16-byte layout alignment), enumerated as units q = tid + b*NT, q < nq
+struct FrameGeo { int x_lo, cs, y_lo, rows, nq, nb; };
+static FrameGeo frame_geo(const Launch &L, const Stage &G, int VW) {
+    FrameGeo f;
+    f.x_lo = -(int)((G.ex0 + VW - 1) / VW * VW);
+    const int x_hi = L.tx + (G.ex1 + VW - 1) / VW * VW;
+    f.cs = (x_hi - f.x_lo) / VW;
+    f.y_lo = -G.ey0;
+    f.rows = L.ty + G.ey0 + G.ey1;
+    f.nq = f.rows * f.cs;
+    f.nb = (f.nq + L.nt - 1) / L.nt;
+    return f;
+}
+
 // registers the generated code keeps live (chooser's occupancy model)
 int codegen_regs(const stencil_program *p, const Launch &L) {
     const int w = p->elem / 4;
     int persistent = 0, transient = 0;
+    if (L.fr) {
+        const int VW = 16 / p->elem;
+        for (const Stage &G : L.st) {
+            if (!G.needed) continue;
+            auto pos = block_positions(L, G);
+            const FrameGeo f = frame_geo(L, G, VW);
+            transient = std::max(transient, ((int)pos.size() + VW) * w * std::min(f.nb, 2));
+            if (G.keep == Keep::Reg) persistent += VW * f.nb * G.depth * w;
+        }
+        return 40 + persistent + transient + 2 * (int)L.in.size();
+    }
     for (const Stage &G : L.st) {
         if (!G.needed) continue;
         auto pos = block_positions(L, G);
@@ -158,7 +185,10 @@ std::string generate_launch(const stencil_program *p, Launch &L, int index, bool
     int XT, YT;
     core_geometry(L, &XT, &YT);
     const int VX = L.vx, VY = L.vy, CBY = L.cby, NPB = VX * VY;
-    if (YT * VY * CBY != L.ty || XT * VX != L.tx || XT * YT != L.nt)
+    const bool FR = L.fr;  // region-vector evaluation (frame mode)
+    if (FR && (VX != VW || VY != 1 || CBY != 1 || L.tx % VW))
+        fail(SP_E_RESOURCES, "internal: frame mode needs 16-byte x-vectors");
+    if (!FR && (YT * VY * CBY != L.ty || XT * VX != L.tx || XT * YT != L.nt))
         fail(SP_E_RESOURCES, "internal: inconsistent block geometry");
     for (const RegionClass &R : L.cls)
         if (R.x0 > 0 || R.x1 < 0 || R.y0 > 0 || R.y1 < 0)
@@ -233,6 +263,10 @@ std::string generate_launch(const stencil_program *p, Launch &L, int index, bool
     // statement coefficients live in constant memory: FP64 FMA/MUL take them as
     // constant-bank operands instead of re-materialising each one per use
     o << "/*SF_COEF_TABLE*/\n}\n";
+    // fp64 coefficients are uniform-register operands of DFMA/DMUL on sm_100 (no constant-bank
+    // operand); fp32 literals are FFMA immediates, so the table only serves fp64
+    const int coef_mode = f32 ? 0 : p->opt.coef_const;
+    const bool cc2 = coef_mode == 2;
     std::map<uint64_t, int> coef_idx;
     std::vector<double> coefs;
     auto coef_ref = [&](double c) {
@@ -243,7 +277,11 @@ std::string generate_launch(const stencil_program *p, Launch &L, int index, bool
             it = coef_idx.emplace(bits, (int)coefs.size()).first;
             coefs.push_back(c);
         }
-        return "SFK[" + num(it->second) + "]";
+        // coef_const 2: the index carries a per-step zero read from constant memory, so the
+        // address is not loop-invariant: ptxas loads each coefficient right before its use
+        // (one LDCU.64 into a uniform register pair) instead of hoisting the whole table into
+        // registers (spills) or materialising each literal with two UMOVs (measured in SASS)
+        return "SFK[" + num(it->second) + (cc2 ? " + sfz" : "") + "]";
     };
     o << "extern \"C\" __global__ void __launch_bounds__(" << L.nth << ", " << std::max(1, p->opt.minblocks)
       << ") " << L.fn
@@ -451,6 +489,10 @@ std::string generate_launch(const stencil_program *p, Launch &L, int index, bool
     // halo tables per class
     std::vector<int> nh(L.cls.size()), hp(L.cls.size());
     for (size_t c = 0; c < L.cls.size(); ++c) {
+        if (FR) {  // every region is covered by x-vectors: no point-wise halo strips
+            nh[c] = hp[c] = 0;
+            continue;
+        }
         const RegionClass &R = L.cls[c];
         const int W = L.tx + R.x1 - R.x0, H = L.ty + R.y1 - R.y0;
         nh[c] = W * H - L.tx * L.ty;
@@ -494,7 +536,8 @@ std::string generate_launch(const stencil_program *p, Launch &L, int index, bool
         if (!G.needed) continue;
         bpos[m] = block_positions(L, G);
         if (G.keep == Keep::Reg) {
-            o << "  T rq" << m << "[CBY][" << NPB << "][" << G.depth << "];\n";
+            o << "  T rq" << m << "[" << (FR ? frame_geo(L, G, VW).nb : CBY) << "][" << NPB << "]["
+              << G.depth << "];\n";
             if (nh[G.cls]) o << "  T rh" << m << "[" << hp[G.cls] << "][" << G.depth << "];\n";
         }
     }
@@ -534,6 +577,7 @@ std::string generate_launch(const stencil_program *p, Launch &L, int index, bool
     // ------------------------------------------------------------- z-march
     for (int r = 0; r < n_ready; ++r) o << "  unsigned cph" << r << " = 0;\n";
     o << "  for (int k = KF; k < zc; ++k) {\n";
+    if (cc2) o << "    const int sfz = SFZ[k & 1];  // always 0 (see coef_ref)\n";
     if (tma) {
         o << "    sf_mbar_wait(&full[(k - KF) & " << NB - 1 << "], ((k - KF) >> " << log2i(NB)
           << ") & 1);\n";
@@ -616,7 +660,7 @@ std::string generate_launch(const stencil_program *p, Launch &L, int index, bool
     bool any_boxed = false;
     for (const Stage &G : L.st)
         if (G.needed && p->stmts[G.gid].boxed) any_boxed = true;
-    const bool spec = (L.fastpath >= 0 ? L.fastpath : p->opt.fastpath) && !any_boxed;
+    const bool spec = (L.fastpath >= 0 ? L.fastpath : p->opt.fastpath) && !any_boxed && !FR;
     if (spec) {
         int kst0 = INT32_MIN;
         int lmin = INT32_MAX, lmax = INT32_MIN, slmin = INT32_MAX, slmax = INT32_MIN;
@@ -660,7 +704,8 @@ std::string generate_launch(const stencil_program *p, Launch &L, int index, bool
           << " depth " << G.depth << "\n";
         // register-stage queues advance every step
         if (G.keep == Keep::Reg && G.depth > 1) {
-            o << "      #pragma unroll\n      for (int b = 0; b < CBY; ++b)\n"
+            o << "      #pragma unroll\n      for (int b = 0; b < " << (FR ? num(frame_geo(L, G, VW).nb) : "CBY")
+              << "; ++b)\n"
               << "      #pragma unroll\n      for (int i = 0; i < " << NPB << "; ++i)\n"
               << "      #pragma unroll\n      for (int d = 0; d < " << G.depth - 1 << "; ++d) rq" << m
               << "[b][i][d] = rq" << m << "[b][i][d + 1];\n";
@@ -672,6 +717,7 @@ std::string generate_launch(const stencil_program *p, Launch &L, int index, bool
         // address of a block position in a layout at plane offset cc
         auto baddr = [&](const PosKey &k, int cc) {
             Lay l{k.stage, k.id};
+            if (FR) return bname(l, cc) + " + fi_" + lname(l) + " + (" + num(k.y * lw(l) + k.x) + ")";
             return bname(l, cc) + " + cb_" + lname(l) + " + b * (YT * VY * " + num(lw(l)) + ") + (" +
                    num(k.y * lw(l) + k.x) + ")";
         };
@@ -725,11 +771,38 @@ std::string generate_launch(const stencil_program *p, Launch &L, int index, bool
         else if (boxed)
             o << "        const bool fast = X0 >= " << BX0 << " && X0 + TX <= " << BX1 << " && Y0 >= "
               << BY0 << " && Y0 + TY <= " << BY1 << " && zin;\n";
-        else
+        else if (FR) {  // the statement's whole (vector-rounded) region is interior
+            const FrameGeo f = frame_geo(L, G, VW);
+            o << "        const bool fast = zin && X0 + (" << f.x_lo << ") >= 0 && X0 + (" << f.x_lo + f.cs * VW
+              << ") <= NX && Y0 + (" << f.y_lo << ") >= 0 && Y0 + (" << f.y_lo + f.rows << ") <= NY;\n";
+        } else
             o << "        const bool fast = tile_in && zin;\n";
 
-        // ---- core blocks
-        o << "        #pragma unroll\n        for (int b = 0; b < CBY; ++b) {\n";
+        // ---- core blocks (frame mode: the region's x-vectors, unit q = tid + b*NT)
+        std::string GX0 = "X0 + xt * VX", GY0 = "Y0 + by", GOFF = "cg + b * (YT * VY * XP)";
+        std::string blk_close = "        }\n";
+        if (FR) {
+            const FrameGeo f = frame_geo(L, G, VW);
+            o << "        #pragma unroll\n        for (int b = 0; b < " << f.nb << "; ++b) {\n";
+            o << "          const int qq = tid + b * NT;\n";
+            if (f.nq % L.nt) {
+                o << "          if (qq < " << f.nq << ") {\n";
+                blk_close = "          }\n        }\n";
+            }
+            o << "          const int fy = " << f.y_lo << " + qq / " << f.cs << ", fx = " << f.x_lo << " + (qq % "
+              << f.cs << ") * " << VW << ";\n";
+            std::set<Lay> used;
+            if (G.keep == Keep::Smem) used.insert(Lay{true, m});
+            for (auto &kv : pos) used.insert(Lay{kv.first.stage, kv.first.id});
+            for (const Lay &l : used)
+                o << "          const int fi_" << lname(l) << " = (fy - (" << ly0(l) << ")) * " << lw(l)
+                  << " + (fx - (" << lx0(l) << "));\n";
+            GX0 = "X0 + fx";
+            GY0 = "Y0 + fy";
+            GOFF = "((Y0 + fy + OYA) * XP + X0 + fx + OXA)";
+        } else {
+            o << "        #pragma unroll\n        for (int b = 0; b < CBY; ++b) {\n";
+        }
         // direct loads, vectorised along x where aligned
         std::map<std::tuple<bool, int, int, int>, std::set<int>> rows;  // (stage,id,c,y) -> xs
         for (auto &kv : pos)
@@ -820,7 +893,7 @@ std::string generate_launch(const stencil_program *p, Launch &L, int index, bool
                 std::string a = opd(t.a);
                 if (t.coef == 1.0) return a;
                 if (t.coef == -1.0) return "(-" + a + ")";
-                return (p->opt.coef_const ? coef_ref(t.coef) : "(T)" + lit(t.coef, f32)) + " * " +
+                return (coef_mode ? coef_ref(t.coef) : "(T)" + lit(t.coef, f32)) + " * " +
                        a;
             };
             std::vector<std::string> part(ACC);
@@ -850,25 +923,32 @@ std::string generate_launch(const stencil_program *p, Launch &L, int index, bool
                 o << "          T o" << iy << "_" << jx << " = "
                   << term_expr([&](const Src &s) { return core_operand(s, iy, jx); }) << ";\n";
         // ghost substitution and store predicates outside the interior (edge tiles, z ghosts)
-        o << "          const int by = (b * YT + yt) * VY;\n";
+        if (!FR) o << "          const int by = (b * YT + yt) * VY;\n";
         o << "          if (!fast) {\n";
         for (int iy = 0; iy < VY; ++iy)
             for (int jx = 0; jx < VX; ++jx) {
-                std::string gx = "X0 + xt * VX + " + num(jx), gy = "Y0 + by + " + num(iy);
-                const std::string inb = boxed ? gx + " >= " + BX0 + " && " + gx + " < " + BX1 +
-                                                    " && " + gy + " >= " + BY0 + " && " + gy + " < " + BY1
-                                              : gx + " < NX && " + gy + " < NY";
+                std::string gx = GX0 + " + " + num(jx), gy = GY0 + " + " + num(iy);
+                std::string inb = boxed ? gx + " >= " + BX0 + " && " + gx + " < " + BX1 +
+                                              " && " + gy + " >= " + BY0 + " && " + gy + " < " + BY1
+                                        : gx + " < NX && " + gy + " < NY";
+                std::string alloc = gx + " < XP - OXA && " + gy + " < YA - OYA";
+                if (FR) {  // region points left of / above the tile as well
+                    inb = gx + " >= 0 && " + gy + " >= 0 && " + inb;
+                    alloc = gx + " + OXA >= 0 && " + gy + " + OYA >= 0 && " + alloc;
+                }
                 o << "            if (!(zin && " << inb << ")) o" << iy << "_"
-                  << jx << " = sf_ldg_pred(gpl + cg + b * (YT * VY * XP) + (" << iy << " * XP + " << jx
-                  << "), zal && " << gx << " < XP - OXA && " << gy << " < YA - OYA);\n";
+                  << jx << " = sf_ldg_pred(gpl + " << GOFF << " + (" << iy << " * XP + " << jx
+                  << "), zal && " << alloc << ");\n";
             }
         o << "          }\n";
         // sinks
         if (G.keep == Keep::Smem) {
             Lay self{true, m};
             for (int iy = 0; iy < VY; ++iy) {
-                std::string a = bname(self, G.lead) + " + cb_" + lname(self) + " + b * (YT * VY * " +
-                                num(lw(self)) + ") + (" + num(iy * lw(self)) + ")";
+                std::string a = FR ? bname(self, G.lead) + " + fi_" + lname(self) + " + (" +
+                                         num(iy * lw(self)) + ")"
+                                   : bname(self, G.lead) + " + cb_" + lname(self) + " + b * (YT * VY * " +
+                                         num(lw(self)) + ") + (" + num(iy * lw(self)) + ")";
                 if (vec_ok) {
                     for (int jx = 0; jx < VX; jx += VW) {
                         o << "          *reinterpret_cast<T2 *>(" << a << " + " << jx << ") = T2{";
@@ -908,7 +988,7 @@ std::string generate_launch(const stencil_program *p, Launch &L, int index, bool
                 o << ind << "} else {\n";
                 for (int iy = 0; iy < VY; ++iy)
                     for (int jx = 0; jx < VX; ++jx) {
-                        const std::string gx = "X0 + xt * VX + " + num(jx), gy = "Y0 + by + " + num(iy);
+                        const std::string gx = GX0 + " + " + num(jx), gy = GY0 + " + " + num(iy);
                         const std::string inb = boxed ? "zin && " + gx + " >= " + BX0 + " && " + gx + " < " +
                                                             BX1 + " && " + gy + " >= " + BY0 + " && " + gy +
                                                             " < " + BY1
@@ -918,8 +998,11 @@ std::string generate_launch(const stencil_program *p, Launch &L, int index, bool
                     }
                 o << ind << "}\n";
             };
-            o << "          if (zst) {\n";
-            o << "            T *const gb = gpl + cg + b * (YT * VY * XP);\n";
+            if (FR)  // frame units inside the tile core (x-vectors are whole: TX % VW == 0)
+                o << "          if (zst && fy >= 0 && fy < TY && fx >= 0 && fx < TX) {\n";
+            else
+                o << "          if (zst) {\n";
+            o << "            T *const gb = gpl + " << GOFF << ";\n";
             stores("gb", "            ");
             for (size_t k = 0; k < L.pushes.size(); ++k) {
                 const Launch::Push &u = L.pushes[k];
@@ -942,7 +1025,7 @@ std::string generate_launch(const stencil_program *p, Launch &L, int index, bool
             }
             o << "          }\n";
         }
-        o << "        }\n";
+        o << blk_close;
 
         // ---- halo points (point-wise)
         if (nh[c]) {
@@ -961,14 +1044,25 @@ std::string generate_launch(const stencil_program *p, Launch &L, int index, bool
             o << "          const int f = h" << c << "_f[i];\n";
             if (CX > 1) o << "          if (f & 48) continue;  // the cluster neighbour computes it\n";
             // ghost points (e.g. the y-halo rows of full-height tiles) are only loaded
-            o << "          T v;\n";
-            if (boxed)
-                o << "          const int hx = h" << c << "_x[i], hy = h" << c << "_y[i];\n"
-                  << "          if (zin && hx >= " << BX0 << " && hx < " << BX1 << " && hy >= " << BY0
-                  << " && hy < " << BY1 << ") v = " << term_expr(halo_operand) << ";\n";
-            else
-                o << "          if (zin && (f & 2)) v = " << term_expr(halo_operand) << ";\n";
-            o << "          else v = sf_ldg_pred(gpl + h" << c << "_g[i], zal && (f & 8));\n";
+            std::string hin;  // the point is evaluated (not a ghost / outside the loop box)
+            if (boxed) {
+                o << "          const int hx = h" << c << "_x[i], hy = h" << c << "_y[i];\n";
+                hin = "zin && hx >= " + BX0 + " && hx < " + BX1 + " && hy >= " + BY0 + " && hy < " + BY1;
+            } else {
+                hin = "zin && (f & 2)";
+            }
+            if (p->opt.halo_sel) {
+                // every halo point's expression is evaluated (its operands are inside the
+                // layouts; a ghost point's value is discarded) and the ghost value replaces
+                // it after: no branch around the loads, so the unrolled points interleave
+                o << "          T v = " << term_expr(halo_operand) << ";\n";
+                o << "          if (" << (FP && !boxed ? "!(f & 2)" : "!(" + hin + ")")
+                  << ") v = sf_ldg_pred(gpl + h" << c << "_g[i], zal && (f & 8));\n";
+            } else {
+                o << "          T v;\n";
+                o << "          if (" << hin << ") v = " << term_expr(halo_operand) << ";\n";
+                o << "          else v = sf_ldg_pred(gpl + h" << c << "_g[i], zal && (f & 8));\n";
+            }
             if (G.keep == Keep::Smem) {
                 Lay self{true, m};
                 o << "          " << bname(self, G.lead) << "[h" << c << "_" << lname(self)
@@ -1054,6 +1148,7 @@ std::string generate_launch(const stencil_program *p, Launch &L, int index, bool
     for (size_t i = 0; i < coefs.size(); ++i) tbl << (i ? ", " : "") << lit(coefs[i], f32);
     if (coefs.empty()) tbl << "0";
     tbl << "};";
+    if (cc2) tbl << "\n__constant__ int SFZ[2];  // zero-initialised module global";
     const std::string marker = "/*SF_COEF_TABLE*/";
     L.source.replace(L.source.find(marker), marker.size(), tbl.str());
     return L.source;

@@ -240,7 +240,10 @@ static void layout_launch(const stencil_program *p, Launch &L) {
     L.rw_pad = 16 / e;  // TMA: inner box extent multiple of 16 B
     L.in_off.clear(); L.in_plane.clear(); L.in_rw.clear(); L.in_rh.clear(); L.in_depth.clear();
     L.st_off.clear(); L.st_plane.clear(); L.st_w.clear(); L.st_h.clear(); L.st_depth.clear();
-    int64_t off = 0;
+    // region-vector evaluation reads up to VW-1+reach elements beyond a layout row's
+    // columns at the region edges (lanes whose results are never consumed): guard bands
+    // keep those reads inside the allocation
+    int64_t off = L.fr ? 256 : 0;
     L.n_bars = 0;
     for (Input &I : L.in) {
         // the innermost start coordinate of a TMA box must be 16-B aligned: the tile
@@ -279,6 +282,7 @@ static void layout_launch(const stencil_program *p, Launch &L) {
             L.st_depth.push_back(0);
         }
     }
+    if (L.fr) off += 256;
     off = rup(off, 8);
     L.bar_off = off;
     off += 8 * (int64_t)L.n_bars;
@@ -369,12 +373,26 @@ static int max_region_points(const Launch &L) {
     return m;
 }
 
+// Region-vector evaluation ("frame"): needs the TMA loader and no per-statement loop
+// boxes; peer push and clusters keep the block form (their codegen assumes it).
+static bool frame_eligible(const stencil_program *p, const Launch &L) {
+    if (p->opt.loader != 0 || p->opt.xpush || p->opt.cluster_x > 1) return false;
+    for (const Stage &G : L.st)
+        if (G.needed && p->stmts[G.gid].boxed) return false;
+    return true;
+}
+
 void choose_config(const stencil_program *p, Launch &L, bool quick) {
     const sp_grid &g = p->grid;
     const int e = p->elem;
     const int64_t nz = g.nz_local;
     const Options &o = p->opt;
-    std::vector<int> cx, cz, cn, cp, cvx, cvy, ccb;
+    L.fr = frame_eligible(p, L) && (L.frame_pin >= 0 ? L.frame_pin != 0 : o.frame != 0);
+    const bool fr = L.fr;
+    const int VW = 16 / e;
+    std::vector<int> cx, cz, cn, cp, cvx, cvy, ccb, cty;
+    if (o.tile_y) cty = {o.tile_y};
+    else cty = {4, 8, 16, 32};
     if (o.tile_x) cx = {o.tile_x};
     else if (quick) cx = e == 8 ? std::vector<int>{32, 64} : std::vector<int>{64, 128};
     else cx = e == 8 ? std::vector<int>{16, 32, 64} : std::vector<int>{32, 64, 128};
@@ -392,6 +410,11 @@ void choose_config(const stencil_program *p, Launch &L, bool quick) {
     else cvy = {1, 2, 4};
     if (o.block_cby) ccb = {o.block_cby};
     else ccb = {1, 2, 4};
+    if (fr) {  // one 16-byte x-vector per evaluation unit; the tile height is free
+        cvx = {VW};
+        cvy = {1};
+        ccb = {1};
+    }
     const double sms = p->num_sms;
     const double clk = 1.85e9;
     const double hbm = 6.0e12, smem_bw = sms * 128 * clk;
@@ -405,21 +428,22 @@ void choose_config(const stencil_program *p, Launch &L, bool quick) {
             if (tx % vx) continue;
             const int xt = tx / vx;
             for (int nt : cn) {
-                if (nt % xt || xt > nt) continue;
-                const int yt = nt / xt;
-                for (int vy : cvy)
+                if (!fr && (nt % xt || xt > nt)) continue;
+                const int yt = fr ? 1 : nt / xt;
+                for (int vy : (fr ? cty : cvy))
                     for (int cby : ccb) {
-                        const int ty = yt * vy * cby;
-                        if (o.tile_y && ty != o.tile_y) continue;
-                        if (!o.tile_y && (ty > 64 || (ty >= 2 * g.ny && (vy > 1 || cby > 1))))
+                        const int ty = fr ? vy : yt * vy * cby;
+                        if (fr && !o.tile_y && ty >= 2 * g.ny && ty != cty.front()) continue;
+                        if (!fr && o.tile_y && ty != o.tile_y) continue;
+                        if (!fr && !o.tile_y && (ty > 64 || (ty >= 2 * g.ny && (vy > 1 || cby > 1))))
                             continue;
                         for (int zc : cz) {
                             if (!o.zchunk && zc >= 2 * nz && zc != cz.front()) continue;
                             for (int pf : cp) {
                                 Launch C = L;
                                 C.tx = tx; C.ty = ty; C.zc = (int)std::min<int64_t>(zc, nz);
-                                C.pf = pf; C.nt = nt; C.vx = vx; C.vy = vy; C.cby = cby;
-                                C.zq = o.zqueue;
+                                C.pf = pf; C.nt = nt; C.vx = vx; C.vy = fr ? 1 : vy; C.cby = cby;
+                                C.zq = fr ? 0 : o.zqueue;
                                 C.nth = nt + (o.loader == 0 ? 32 : 0);
                                 layout_launch(p, C);
                                 if (C.smem > 227 * 1024) continue;
@@ -461,7 +485,7 @@ void choose_config(const stencil_program *p, Launch &L, bool quick) {
                                 double t_sm = C.smem_pt * pts / (smem_bw * 0.8);
                                 double t_alu = C.flops_exec * pts / alu;
                                 const double warps = res * nt / 32;
-                                const double ilp = std::min(4, vx * vy * cby);
+                                const double ilp = fr ? 4.0 : std::min(4, vx * vy * cby);
                                 const double ipc = std::min(3.2, warps * std::sqrt(ilp) / 16.0);
                                 double t_issue = estimate_instr(C, p->opt.fmad && p->opt.factor) * pts /
                                                  32.0 / (sms * ipc * clk);
@@ -550,6 +574,7 @@ void analyze_mode(stencil_program *p, bool fused, const std::vector<std::vector<
             fail(SP_E_RESOURCES, L.name + ": accumulated z-reach " +
                                      std::to_string(std::max(L.z_below, L.z_above)) +
                                      " exceeds zhalo " + std::to_string(p->grid.zhalo));
+        if (!fused) L.frame_pin = 0;  // the "frame" option applies to fused groups (pins to any)
         if (!L.dead) {
             // per-launch tuned configuration (sp_plan_tune) overrides the chooser's search
             auto &tune = fused ? p->tune_fused : p->tune_unfused;
@@ -567,6 +592,7 @@ void analyze_mode(stencil_program *p, bool fused, const std::vector<std::vector<
                 if (c.block_cby) p->opt.block_cby = c.block_cby;
                 if (c.zqueue) p->opt.zqueue = c.zqueue - 1;
                 if (c.fastpath) L.fastpath = c.fastpath - 1;
+                if (c.frame) L.frame_pin = c.frame - 1;
                 try {
                     choose_config(p, L);
                 } catch (...) {

@@ -85,6 +85,7 @@ class Objective {
                 if (pin->block_cby) p_->opt.block_cby = pin->block_cby;
                 if (pin->zqueue) p_->opt.zqueue = pin->zqueue - 1;
                 if (pin->fastpath) L.fastpath = pin->fastpath - 1;
+                if (pin->frame) L.frame_pin = pin->frame - 1;
             }
             choose_config(p_, L, quick);
             p_->opt = saved;
@@ -154,6 +155,7 @@ class MeasuredObjective : public Objective {
                 c.tile_x = L.tx; c.tile_y = L.ty; c.zchunk = L.zc; c.threads = L.nt; c.prefetch = L.pf;
                 c.block_x = L.vx; c.block_y = L.vy; c.block_cby = L.cby;
                 c.fastpath = L.fastpath >= 0 ? L.fastpath + 1 : 0;
+                c.frame = L.fr ? 2 : 1;
                 bool dup = false;
                 for (const auto &o : owner)
                     dup |= o.first == i && !std::memcmp(&o.second, &c, sizeof c);

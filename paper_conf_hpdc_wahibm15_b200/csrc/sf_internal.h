@@ -40,7 +40,8 @@ struct Options {
     int suspend_hint = 0;  // ns hint of mbarrier.try_wait (0 = none)
     int l2pf = 1;          // TMA L2 prefetch distance in steps beyond the ring (0 = off;
                            // r1s3: 1 wins with the prefetch-1 rings: C2 -3.4 %, C5 -2 %, C4 -0.7 %)
-    int coef_const = 0;    // 1: coefficients in a __constant__ table (r1: 35 % slower)
+    int coef_const = 0;    // fp64: 1 = __constant__ table (r1: 35 % slower, hoisted), 2 = table read
+                           // per use through a per-step zero (one LDCU.64 per coefficient)
     int pdl = 1;        // programmatic dependent launch: 1 = fused groups, 2 = all, 0 = off
     int acc_split = 1;  // >1: interleaved partial sums in the perf build (no gain measured r1)
     int factor = 1;     // perf build: terms sharing one b operand are summed, then multiplied once
@@ -52,6 +53,9 @@ struct Options {
                        // overflows the 32 KB instruction cache: C4 +2 %, C2 +12 % slower)
     int minblocks = 1; // __launch_bounds__ minimum resident CTAs (register budget for ptxas)
     int cluster_x = 1; // > 1: CTAs per cluster along x sharing x-halos of smem stages over DSMEM
+    int frame = 0;     // region-vector evaluation of fused launches (see stencilfuse.h "frame")
+    int halo_sel = 0;  // halo points: expression always evaluated, ghost value selected after
+                       // (no branch around the loads: several halo points' loads interleave)
     int regcap = 1; // recompile a few registers tighter when that adds a resident CTA:
                     // 0 never, 1 peer-push kernels, 2 every kernel
 };
@@ -143,6 +147,8 @@ struct Launch {
     bool dead = false;       // nothing to compute (all stages dead)
     bool pdl = false;        // launched with programmatic stream serialization
     int fastpath = -1;       // per-launch pin of the "fastpath" codegen variant (-1: option)
+    int frame_pin = -1;      // per-launch pin of the "frame" evaluation mode (-1: option)
+    bool fr = false;         // region-vector evaluation (resolved from pin/option/eligibility)
 };
 
 struct Mode {

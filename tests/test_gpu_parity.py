@@ -13,6 +13,7 @@ import numpy as np
 import pytest
 
 from _harness import assert_close, gpu_run, oracle_outputs, rel_err
+from paper_conf_hpdc_wahibm15_b200 import StencilError
 from synth import programs as P
 
 pytestmark = pytest.mark.gpu
@@ -356,3 +357,38 @@ def test_degenerate_grids_bitexact(cuda_device, n):
         for plan in plans:
             got = gpu_run(prog, "fused", 13, options={"fmad": 0}, plan=prog["plans"][plan], poison=False)
             assert_close(prog, got, ref, exact=True)
+
+
+# Region-vector evaluation (option "frame"): every statement on its whole extended
+# region in 16-byte x-vectors enumerated over the threads.  Tile shapes are free
+# (tile_y independent of threads); ragged grids exercise edge tiles, partial last
+# units (qq < nq) and ghost substitution on halo rows/columns left of / above the tile.
+FRAME_TILES = [{}, dict(tile_x=16, tile_y=3, zchunk=2, threads=32),
+               dict(tile_x=32, tile_y=16, zchunk=7, threads=128, prefetch=1),
+               dict(tile_x=64, tile_y=8, zchunk=5, threads=256, prefetch=2)]
+
+
+@pytest.mark.parametrize("name,prog,plans", CASES, ids=[c[0] for c in CASES])
+@pytest.mark.parametrize("fmad", [0, 1])
+def test_frame_mode_parity(cuda_device, name, prog, plans, fmad):
+    """frame=1: fused plans (complex fusion with halo recompute, fission+fusion) match
+    the oracle bit-exactly in the parity build and within R17 in the perf build."""
+    ref = oracle_outputs(prog, seed=12)
+    for tiles in FRAME_TILES:
+        for plan in plans:
+            try:
+                got = gpu_run(prog, "fused", 12, options=dict(tiles, fmad=fmad, frame=1),
+                              plan=prog["plans"][plan])
+            except StencilError as e:  # a pinned tile whose rings exceed shared memory
+                assert tiles and e.code == 6, e
+                continue
+            assert_close(prog, got, ref, exact=fmad == 0)
+
+
+def test_frame_mode_c4_reduced_bitexact(cuda_device):
+    """frame=1 on the SCALE-LES-shaped 40-kernel DAG (reduced grid), bit-exact."""
+    prog = _c4_small()
+    ref = oracle_outputs(prog, seed=13)
+    for tiles in ({}, dict(tile_x=32, tile_y=5, zchunk=4, threads=64)):
+        got = gpu_run(prog, "fused", 13, options=dict(tiles, fmad=0, frame=1), plan=prog["plans"]["fused"])
+        assert_close(prog, got, ref, exact=True)

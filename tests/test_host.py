@@ -624,3 +624,27 @@ def test_live_out_stores_writer_before_boxed_rewrite():
     assert p.report("fused", 0)["n_stores"] == 1
     p.set_plan([["K1"], ["K2"], ["K3"]])
     assert [r["n_stores"] for r in p.reports("fused")] == [1, 1, 1]
+
+
+@pytest.mark.parametrize("name", ["C2", "C3", "C5"])
+def test_frame_mode_codegen_and_pins(name):
+    """Option / pin "frame": region-vector evaluation replaces the point-wise halo strips
+    (no per-thread halo tables in the source), units are 16-byte x-vectors, the tile
+    height is free of the thread count, and the kernels compile for sm_100a."""
+    prog = P.CONFIGS[name]()
+    plan = prog["plans"]["fission_fused" if name == "C3" else "fused"]
+    p = Program(prog, options={"frame": 1})
+    p.set_plan(plan)
+    src = p.source("fused")
+    assert "fi_" in src and "_f[i]" not in src
+    vw = 16 // (4 if prog["dtype"] == "f32" else 8)
+    assert all(r["block_x"] == vw and r["block_y"] == 1 for r in p.reports("fused"))
+    p.compile("fused")
+    assert all(0 < r["regs_per_thread"] <= 255 for r in p.reports("fused"))
+    # a per-launch pin with a tile height no block geometry could give
+    p.tune("fused", 0, dict(tile_x=32, tile_y=5, threads=64, zchunk=8, frame=1))
+    r = p.report("fused", 0)
+    assert (r["tile_x"], r["tile_y"], r["threads"]) == (32, 5, 64)
+    # and the pin can switch it off again for that launch only
+    p.tune("fused", 0, dict(frame=0))
+    assert "_f[i]" in p.source("fused")

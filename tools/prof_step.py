@@ -21,12 +21,19 @@ ap.add_argument("--warmup", type=int, default=1)
 ap.add_argument("--unfused", action="store_true")
 ap.add_argument("--opt", action="append", default=[])
 ap.add_argument("--plan", default="fused")
+ap.add_argument("--cfg", help="per-launch pins (tools/frame_tune.py --out) instead of the bench's")
 a = ap.parse_args()
 prog = bench.load_workload(a.workload)
 opts = {kv.split("=")[0]: int(kv.split("=")[1]) for kv in a.opt}
 p = Program(prog, options=opts)
 p.set_plan(bench.plan_of(prog, a.plan))
-bench.apply_tuning(p, prog, a.plan)
+if a.cfg:
+    import json
+    for i, c in enumerate(json.load(open(a.cfg))["configs"]):
+        if c:
+            p.tune("fused", i, c)
+else:
+    bench.apply_tuning(p, prog, a.plan)
 dev = torch.device("cuda:0")
 p.allocate(dev, fill=0.0)
 bench.fill_inputs(p, prog, dev, 0, prog["grid"]["ghost"][2])

@@ -476,7 +476,21 @@ std::string generate_launch(const stencil_program *p, Launch &L, int index, bool
         o << "  const int cb_" << lname(l) << " = (yt * VY - (" << ly0(l) << ")) * " << lw(l)
           << " + (xt * VX - (" << lx0(l) << "));\n";
     o << "  const int cg = (Y0 + yt * VY + OYA) * XP + X0 + xt * VX + OXA;\n";
-    o << "  const bool tile_in = X0 + TX <= NX && Y0 + TY <= NY;  // all core points interior\n";
+    if (FR) {  // frame mode: every statement's (vector-rounded) region is interior
+        int mx0 = 0, mx1 = 0, my0 = 0, my1 = 0;
+        for (const Stage &G : L.st) {
+            if (!G.needed) continue;
+            const FrameGeo f = frame_geo(L, G, VW);
+            mx0 = std::max(mx0, -f.x_lo);
+            mx1 = std::max(mx1, f.x_lo + f.cs * VW - L.tx);
+            my0 = std::max(my0, -f.y_lo);
+            my1 = std::max(my1, f.y_lo + f.rows - L.ty);
+        }
+        o << "  const bool tile_in = X0 >= " << mx0 << " && X0 + TX + " << mx1 << " <= NX && Y0 >= " << my0
+          << " && Y0 + TY + " << my1 << " <= NY;  // all regions interior\n";
+    } else {
+        o << "  const bool tile_in = X0 + TX <= NX && Y0 + TY <= NY;  // all core points interior\n";
+    }
 
     // statement loop bounds (reading R2'): local-coordinate box of a boxed stage
     std::set<int> box_cls;
@@ -607,17 +621,24 @@ std::string generate_launch(const stencil_program *p, Launch &L, int index, bool
         for (int c = kv.second.cmin; c <= kv.second.cmax; ++c)
             basekeys.insert({Lay{false, kv.first.id}, c});
     auto bname = [&](const Lay &l, int c) { return "B" + lname(l) + "_" + sg(c); };
+    // ring slot of plane k + c in a ring whose slot 0 holds plane lo: (k + c - lo) mod D,
+    // shifted by a multiple of D so the operand is non-negative for every step k >= KF
+    // (an unsigned modulo: a mask or a multiply-high instead of the signed sequence)
+    auto uslot = [&](int c, int lo, int D) {
+        const int need = lo - c - L.kfirst;
+        const int M = need > 0 ? (need + D - 1) / D : 0;
+        return "((unsigned)(k + (" + num(c - lo + D * M) + ")) % " + num(D) + "u)";
+    };
     for (auto &bk : basekeys) {
         const Lay &l = bk.first;
         const int c = bk.second;
         std::string slot;
         int64_t plane;
         if (l.stage) {
-            slot = "((k + (" + num(c) + ") - (" + num(L.st[l.id].loff) + ")) % " +
-                   num(L.st_depth[l.id]) + ")";
+            slot = uslot(c, L.st[l.id].loff, L.st_depth[l.id]);
             plane = L.st_plane[l.id];
         } else {
-            slot = slot_of(l.id, "(k + (" + num(c) + "))");
+            slot = uslot(c, L.in[l.id].qlo, L.in_depth[l.id]);
             plane = L.in_plane[l.id];
         }
         o << "    T *const " << bname(l, c) << " = " << (l.stage ? "st" : "in") << l.id << " + " << slot
@@ -660,7 +681,7 @@ std::string generate_launch(const stencil_program *p, Launch &L, int index, bool
     bool any_boxed = false;
     for (const Stage &G : L.st)
         if (G.needed && p->stmts[G.gid].boxed) any_boxed = true;
-    const bool spec = (L.fastpath >= 0 ? L.fastpath : p->opt.fastpath) && !any_boxed && !FR;
+    const bool spec = (L.fastpath >= 0 ? L.fastpath : p->opt.fastpath) && !any_boxed;
     if (spec) {
         int kst0 = INT32_MIN;
         int lmin = INT32_MAX, lmax = INT32_MIN, slmin = INT32_MAX, slmax = INT32_MIN;

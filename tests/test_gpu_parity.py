@@ -364,8 +364,9 @@ def test_degenerate_grids_bitexact(cuda_device, n):
 # (tile_y independent of threads); ragged grids exercise edge tiles, partial last
 # units (qq < nq) and ghost substitution on halo rows/columns left of / above the tile.
 FRAME_TILES = [{}, dict(tile_x=16, tile_y=3, zchunk=2, threads=32),
-               dict(tile_x=32, tile_y=16, zchunk=7, threads=128, prefetch=1),
-               dict(tile_x=64, tile_y=8, zchunk=5, threads=256, prefetch=2)]
+               dict(tile_x=32, tile_y=16, zchunk=7, threads=128, prefetch=1, fastpath=1),
+               dict(tile_x=64, tile_y=8, zchunk=5, threads=256, prefetch=2),
+               dict(tile_x=32, tile_y=4, zchunk=9, threads=64, fastpath=1)]
 
 
 @pytest.mark.parametrize("name,prog,plans", CASES, ids=[c[0] for c in CASES])

@@ -251,7 +251,9 @@ static void layout_launch(const stencil_program *p, Launch &L) {
         I.bx0 = (int)rup(std::max(I.ex0, 0), L.rw_pad);
         int rw = (int)rup(L.tx + I.bx0 + std::max(I.ex1, 0), L.rw_pad);
         int rh = L.ty + I.ey0 + I.ey1;
-        int64_t plane = rup((int64_t)rw * rh, 128 / e);
+        // frame mode: a 128-B guard after every plane slot (never written) takes the
+        // reads of edge lanes past a row end, so they never touch a slot being refilled
+        int64_t plane = rup((int64_t)rw * rh, 128 / e) + (L.fr ? 128 / e : 0);
         int D = I.ahi - I.alo + 1 + L.pf;  // ring slot = plane mod D (constant modulo per step)
         L.in_off.push_back(off);
         L.in_plane.push_back(plane);
@@ -271,7 +273,7 @@ static void layout_launch(const stencil_program *p, Launch &L) {
         if (G.keep == Keep::Smem) {
             // one plane deeper than the reuse distance: no end-of-step barrier needed
             int D = G.depth + 1;
-            int64_t plane = rup((int64_t)w * h, 128 / e);
+            int64_t plane = rup((int64_t)w * h, 128 / e) + (L.fr ? 128 / e : 0);
             L.st_off.push_back(off);
             L.st_plane.push_back(plane);
             L.st_depth.push_back(D);

@@ -1,6 +1,6 @@
 """Workload for compute-sanitizer runs (tests/test_gpu_sanitizer.py): small C1, C2,
-chain3 and C4 programs, unfused and fused (parity build), each checked bit-exact
-against the oracle.  Usage: python tests/_sanitize_case.py [case ...]"""
+chain3, C3 and C4 programs, unfused and fused (parity build; fused also in the
+region-vector "frame" form), each checked bit-exact against the oracle.  Usage: python tests/_sanitize_case.py [case ...]"""
 import json
 import os
 import sys
@@ -28,6 +28,11 @@ def main(names):
         ref = oracle_outputs(prog, seed=3)
         for mode in ("unfused", "fused"):
             got = gpu_run(prog, mode, 3, options={"fmad": 0}, plan=prog["plans"][plan])
+            assert_close(prog, got, ref, exact=True)
+        # region-vector (frame) form: edge lanes read past row ends into the plane guards
+        for opts in ({"frame": 1}, {"frame": 1, "tile_x": 16, "tile_y": 3, "threads": 64, "zchunk": 2},
+                     {"frame": 1, "fastpath": 1}):
+            got = gpu_run(prog, "fused", 3, options=dict(opts, fmad=0), plan=prog["plans"][plan])
             assert_close(prog, got, ref, exact=True)
         print(f"{name}: ok", flush=True)
 

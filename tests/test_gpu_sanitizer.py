@@ -36,6 +36,10 @@ def test_compute_sanitizer(cuda_device, tool):
     r = subprocess.run(cmd, capture_output=True, text=True, timeout=1500, cwd=ROOT)
     out = r.stdout + r.stderr
     print(out[-3000:])
+    if r.returncode == 86 and "closed on this pool" in out:
+        # the GPU pool's operators closed compute-sanitizer (it wraps the binary and exits 86
+        # without running anything); the last runs are kept in profiles/r2_sanitizer.log
+        pytest.skip("compute-sanitizer closed on this GPU pool: " + out.strip().splitlines()[-1][:200])
     assert r.returncode == 0, out[-6000:]
     assert ("ERROR SUMMARY: 0 errors" in out or "(0 errors, 0 warnings)" in out), out[-6000:]
     for name in ("C1", "C2", "chain3", "C3", "C4"):

@@ -27,13 +27,20 @@ TILES = [{}, dict(tile_x=16, tile_y=2, threads=32, block_x=1, block_y=1, block_c
          dict(tile_x=64, tile_y=8, threads=64, block_x=4, block_y=2, block_cby=1, zchunk=2, prefetch=2)]
 
 
-def single(seed, boxes):
+# region-vector (frame) evaluation: tile_y is free of the thread count
+FRAME_TILES = [dict(frame=1), dict(frame=1, tile_x=16, tile_y=3, threads=32, zchunk=2),
+               dict(frame=1, tile_x=32, tile_y=5, threads=64, zchunk=3, fastpath=1),
+               dict(frame=1, tile_x=64, tile_y=8, threads=256, zchunk=4, prefetch=2)]
+
+
+def single(seed, boxes, frame=False):
     from _fuzz import fuzz_case
     from _harness import assert_close, gpu_run, oracle_outputs
     prog, plans, _, _ = fuzz_case(seed, boxes)
     rng = np.random.default_rng(seed)
     ref = oracle_outputs(prog, seed=seed, poison=False)
-    opts = dict(TILES[int(rng.integers(0, len(TILES)))], fmad=0)
+    tiles = FRAME_TILES if frame else TILES
+    opts = dict(tiles[int(rng.integers(0, len(tiles)))], fmad=0)
     assert_close(prog, gpu_run(prog, "unfused", seed, options=opts, poison=False), ref, exact=True)
     for plan in plans:
         got = gpu_run(prog, "fused", seed, options=opts, plan=plan, poison=False)
@@ -119,6 +126,7 @@ def main():
     ap.add_argument("--seeds", type=int, default=200)
     ap.add_argument("--start", type=int, default=1000)
     ap.add_argument("--ranks", type=int, default=0)
+    ap.add_argument("--frame", action="store_true", help="fused plans in region-vector (frame) mode")
     a = ap.parse_args()
     fails = 0
     for seed in range(a.start, a.start + a.seeds):
@@ -127,12 +135,13 @@ def main():
                 if a.ranks:
                     multi(seed, boxes, a.ranks)
                 else:
-                    single(seed, boxes)
+                    single(seed, boxes, a.frame)
             except Exception:  # noqa: BLE001
                 fails += 1
                 print(f"FAIL seed {seed} boxes {boxes}: {traceback.format_exc().splitlines()[-1][:300]}",
                       flush=True)
-    print(f"fuzz campaign ranks={a.ranks}: {2 * a.seeds} cases, {fails} failures", flush=True)
+    print(f"fuzz campaign ranks={a.ranks} frame={int(a.frame)}: {2 * a.seeds} cases, {fails} failures",
+          flush=True)
 
 
 if __name__ == "__main__":

@@ -1,5 +1,9 @@
 """Peer-push multi-rank step on ONE GPU under MPS (dev tool; a proxy, not a scaling number).
 
+DO NOT RUN on the shared B200 pool: its kernels wait on kernels of other processes on the
+same GPU, which has no co-residency guarantee (the pool's driver recorded Xid 109
+context-switch timeouts for exactly this); kept for reference with its round-1 results.
+
 python tools/mps_xpush.py [--workload C4] [--ranks 2] [--steps 10] [--no-mps]
 
 Starts an MPS daemon (CUDA_MPS_PIPE_DIRECTORY under /tmp), so that the P rank

@@ -48,7 +48,23 @@ CANDIDATES += [dict(c, fastpath=1) for c in list(CANDIDATES)]
 CANDIDATES_F32 += [dict(c, fastpath=1) for c in list(CANDIDATES_F32)]
 
 
-def measured_search(workload, generations=12, population=16, seed=1, candidates=None, reps=3):
+# region-vector (frame) evaluation: the shapes tools/frame_tune.py picked for the C2/C3/C5 groups
+CANDIDATES_FRAME_F32 = [
+    dict(tile_x=32, tile_y=16, threads=256, zchunk=64, prefetch=2, frame=1),
+    dict(tile_x=32, tile_y=32, threads=256, zchunk=32, prefetch=1, frame=1),
+    dict(tile_x=32, tile_y=16, threads=256, zchunk=32, prefetch=1, frame=1),
+    dict(tile_x=64, tile_y=8, threads=256, zchunk=32, prefetch=1, frame=1),
+    dict(tile_x=32, tile_y=16, threads=128, zchunk=32, prefetch=2, frame=1),
+]
+CANDIDATES_FRAME_F64 = [
+    dict(tile_x=32, tile_y=8, threads=128, zchunk=8, prefetch=1, frame=1),
+    dict(tile_x=16, tile_y=16, threads=128, zchunk=32, prefetch=1, frame=1),
+    dict(tile_x=32, tile_y=16, threads=128, zchunk=16, prefetch=1, frame=1),
+]
+
+
+def measured_search(workload, generations=12, population=16, seed=1, candidates=None, reps=3,
+                    frame=False):
     """Run the search on a full-size instance of the workload; returns the plan-file dict."""
     import torch
     import bench
@@ -56,6 +72,8 @@ def measured_search(workload, generations=12, population=16, seed=1, candidates=
     prog = bench.load_workload(workload)
     if candidates is None:
         candidates = CANDIDATES + (CANDIDATES_F32 if prog["dtype"] == "f32" else [])
+        if frame:
+            candidates += CANDIDATES_FRAME_F32 if prog["dtype"] == "f32" else CANDIDATES_FRAME_F64
     dev = torch.device("cuda:0")
     p = Program(prog)
     p.allocate(dev, fill=0.0)
@@ -84,8 +102,10 @@ def main():
     ap.add_argument("--generations", type=int, default=12)
     ap.add_argument("--population", type=int, default=16)
     ap.add_argument("--seed", type=int, default=1)
+    ap.add_argument("--frame", action="store_true", help="add region-vector (frame) candidates")
+    ap.add_argument("--name", default="searched", help="plan name written into C2/C3/C5 plan files")
     a = ap.parse_args()
-    out = measured_search(a.workload, a.generations, a.population, a.seed)
+    out = measured_search(a.workload, a.generations, a.population, a.seed, frame=a.frame)
     print(json.dumps(out["search_report"]), f"{out['search_seconds']:.0f} s")
     for g, c in zip(out["groups"], out["configs"]):
         print(g, c)
@@ -93,7 +113,7 @@ def main():
         if a.workload != "C4" and os.path.exists(a.out):
             # C2/C3/C5 plan files hold named plans: add / replace the "searched" entry
             pj = json.load(open(a.out))
-            pj.setdefault("plans", {})["searched"] = {"groups": out["groups"], "configs": out["configs"],
+            pj.setdefault("plans", {})[a.name] = {"groups": out["groups"], "configs": out["configs"],
                                                       "planner": out["planner"],
                                                       "search_report": out["search_report"]}
             out = pj

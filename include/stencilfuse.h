@@ -239,7 +239,11 @@ sp_status stencil_program_bind(stencil_program *prog, int32_t array, void *dev_p
  *               fusion, §5.5.3) in 16-byte x-vectors of adjacent points
  *               enumerated linearly over the threads, instead of register blocks on
  *               the tile plus point-wise halo strips; launches with loop-bounded
- *               statements, peer push or clusters keep the block form; default 0
+ *               statements, peer push or clusters keep the block form; default 0.
+ *               2: the same with ONE unit grid for all statements of a launch (the
+ *               union of their regions; a statement skips units outside its own), so a
+ *               unit's values at the unit's own position — centre and vertical taps — are
+ *               kept in per-thread register queues instead of re-read from shared memory
  *   "cluster_x" 2..8: fused launches with a shared-memory stage extended in x run as
  *               thread-block clusters of that many x-neighbouring tiles; the x-halo
  *               columns a stage needs inside a neighbour's tile are read from that
@@ -292,7 +296,8 @@ typedef struct {
     int32_t tile_x, tile_y, zchunk, threads, prefetch, block_x, block_y, block_cby;
     int32_t zqueue;
     int32_t fastpath;  /* 0 = the program's "fastpath" option, 1 = off, 2 = on (this launch) */
-    int32_t frame;     /* 0 = the program's "frame" option, 1 = off, 2 = on (this launch) */
+    int32_t frame;     /* 0 = the program's "frame" option, 1 = off, 2 = on, 3 = on with
+                          position-stable units and register z-reuse (this launch) */
 } sp_tile_config;
 
 /* Lazy-fission plan search (the paper's search step,

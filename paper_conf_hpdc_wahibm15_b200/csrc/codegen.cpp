@@ -89,7 +89,7 @@ static std::map<PosKey, PosInfo> block_positions(const Launch &L, const Stage &G
         for (int w = 0; w < 2; ++w) {
             if (w == 1 && !t.has_b) continue;
             const Src &s = w ? t.b : t.a;
-            if (s.stage && L.st[s.idx].keep == Keep::Reg) continue;
+            if (s.stage && (L.st[s.idx].keep == Keep::Reg || (L.fr2 && s.dx == 0 && s.dy == 0))) continue;
             for (int iy = 0; iy < L.vy; ++iy)
                 for (int jx = 0; jx < L.vx; ++jx) {
                     int c = G.lead + s.dz;
@@ -118,6 +118,32 @@ static FrameGeo frame_geo(const Launch &L, const Stage &G, int VW) {
     return f;
 }
 
+// frame mode 2: one unit grid for the whole launch, the union of the statements' regions
+static FrameGeo launch_frame(const Launch &L, int VW) {
+    int x0 = 0, x1 = L.tx, y0 = 0, y1 = L.ty;
+    for (const Stage &G : L.st) {
+        if (!G.needed) continue;
+        const FrameGeo f = frame_geo(L, G, VW);
+        x0 = std::min(x0, f.x_lo);
+        x1 = std::max(x1, f.x_lo + f.cs * VW);
+        y0 = std::min(y0, f.y_lo);
+        y1 = std::max(y1, f.y_lo + f.rows);
+    }
+    FrameGeo f;
+    f.x_lo = x0;
+    f.cs = (x1 - x0) / VW;
+    f.y_lo = y0;
+    f.rows = y1 - y0;
+    f.nq = f.rows * f.cs;
+    f.nb = (f.nq + L.nt - 1) / L.nt;
+    return f;
+}
+// a stage keeps a register queue of its own-position values: register stages always,
+// shared-memory stages too in frame mode 2 (their centre / vertical taps)
+static bool has_rq(const Launch &L, const Stage &G) {
+    return G.keep == Keep::Reg || (L.fr2 && G.keep == Keep::Smem);
+}
+
 // registers the generated code keeps live (chooser's occupancy model)
 int codegen_regs(const stencil_program *p, const Launch &L) {
     const int w = p->elem / 4;
@@ -127,9 +153,25 @@ int codegen_regs(const stencil_program *p, const Launch &L) {
         for (const Stage &G : L.st) {
             if (!G.needed) continue;
             auto pos = block_positions(L, G);
-            const FrameGeo f = frame_geo(L, G, VW);
+            const FrameGeo f = L.fr2 ? launch_frame(L, VW) : frame_geo(L, G, VW);
             transient = std::max(transient, ((int)pos.size() + VW) * w * std::min(f.nb, 2));
-            if (G.keep == Keep::Reg) persistent += VW * f.nb * G.depth * w;
+            if (has_rq(L, G)) persistent += VW * f.nb * G.depth * w;
+        }
+        if (L.fr2) {  // step-wide input queues of the own-position columns
+            const FrameGeo F = launch_frame(L, VW);
+            std::map<int, std::pair<int, int>> rng;
+            for (const Stage &G : L.st) {
+                if (!G.needed) continue;
+                for (auto &kv : block_positions(L, G))
+                    if (!kv.first.stage && kv.first.y == 0 && kv.first.x == 0) {
+                        auto it = rng.emplace(kv.first.id, std::make_pair(kv.second.cmin, kv.second.cmax)).first;
+                        it->second.first = std::min(it->second.first, kv.second.cmin);
+                        it->second.second = std::max(it->second.second, kv.second.cmax);
+                    }
+            }
+            for (auto &kv : rng)
+                if (kv.second.second > kv.second.first)
+                    persistent += VW * F.nb * (kv.second.second - kv.second.first + 1) * w;
         }
         return 40 + persistent + transient + 2 * (int)L.in.size();
     }
@@ -186,6 +228,8 @@ std::string generate_launch(const stencil_program *p, Launch &L, int index, bool
     core_geometry(L, &XT, &YT);
     const int VX = L.vx, VY = L.vy, CBY = L.cby, NPB = VX * VY;
     const bool FR = L.fr;  // region-vector evaluation (frame mode)
+    const bool FR2 = FR && L.fr2;  // ... with one unit grid and register z-reuse
+    const FrameGeo FF = FR ? launch_frame(L, VW) : FrameGeo{};
     if (FR && (VX != VW || VY != 1 || CBY != 1 || L.tx % VW))
         fail(SP_E_RESOURCES, "internal: frame mode needs 16-byte x-vectors");
     if (!FR && (YT * VY * CBY != L.ty || XT * VX != L.tx || XT * YT != L.nt))
@@ -549,8 +593,8 @@ std::string generate_launch(const stencil_program *p, Launch &L, int index, bool
         const Stage &G = L.st[m];
         if (!G.needed) continue;
         bpos[m] = block_positions(L, G);
-        if (G.keep == Keep::Reg) {
-            o << "  T rq" << m << "[" << (FR ? frame_geo(L, G, VW).nb : CBY) << "][" << NPB << "]["
+        if (has_rq(L, G)) {
+            o << "  T rq" << m << "[" << (FR2 ? FF.nb : FR ? frame_geo(L, G, VW).nb : CBY) << "][" << NPB << "]["
               << G.depth << "];\n";
             if (nh[G.cls]) o << "  T rh" << m << "[" << hp[G.cls] << "][" << G.depth << "];\n";
         }
@@ -570,12 +614,27 @@ std::string generate_launch(const stencil_program *p, Launch &L, int index, bool
                 }
         for (auto it = gq.begin(); it != gq.end();)
             it = it->second.cmax > it->second.cmin ? std::next(it) : gq.erase(it);
+        if (FR2) {
+            // frame mode 2 refills a unit's whole x-vector per plane: every lane of an input
+            // with a queued lane gets the union plane range (taps with dx != 0 reach some
+            // lanes of the own vector, so lanes differ in the planes they are read at)
+            std::map<int, PosInfo> un;
+            for (auto &kv : gq) {
+                PosInfo &u = un[kv.first.id];
+                u.cmin = std::min(u.cmin, kv.second.cmin);
+                u.cmax = std::max(u.cmax, kv.second.cmax);
+            }
+            gq.clear();
+            for (auto &kv : un)
+                for (int x = 0; x < VW; ++x) gq[PosKey{false, kv.first, 0, x, 0}] = kv.second;
+        }
     }
     auto gqname = [&](const PosKey &k) {
         return "zg_I" + num(k.id) + "_" + sg(k.y) + "_" + sg(k.x);
     };
     for (auto &kv : gq)
-        o << "  T " << gqname(kv.first) << "[CBY][" << kv.second.cmax - kv.second.cmin + 1 << "];\n";
+        o << "  T " << gqname(kv.first) << "[" << (FR2 ? num(FF.nb) : "CBY") << "]["
+          << kv.second.cmax - kv.second.cmin + 1 << "];\n";
     if (L.zq == 1)
         for (size_t m = 0; m < L.st.size(); ++m)
             for (auto &kv : bpos[m])
@@ -644,7 +703,51 @@ std::string generate_launch(const stencil_program *p, Launch &L, int index, bool
         o << "    T *const " << bname(l, c) << " = " << (l.stage ? "st" : "in") << l.id << " + " << slot
           << " * " << plane << ";\n";
     }
-    if (!gq.empty()) {
+    if (!gq.empty() && FR2) {
+        // frame mode 2: every thread refills the own-position columns of its units (one
+        // 16-byte vector per input and unit: all VW lanes share the plane range) — units
+        // outside an input's loaded box keep stale values nobody reads
+        std::map<int, std::pair<int, int>> cols;  // input -> plane range of its queues
+        for (auto &kv : gq) cols[kv.first.id] = {kv.second.cmin, kv.second.cmax};
+        for (auto &kv : gq)
+            if (kv.second.cmin != cols[kv.first.id].first || kv.second.cmax != cols[kv.first.id].second)
+                fail(SP_E_RESOURCES, "internal: frame-2 input queue lanes differ in plane range");
+        o << "    #pragma unroll\n    for (int b = 0; b < " << FF.nb << "; ++b) {\n";
+        o << "      const int qq = tid + b * NT;\n";
+        o << "      const int fy = " << FF.y_lo << " + qq / " << FF.cs << ", fx = " << FF.x_lo << " + (qq % "
+          << FF.cs << ") * " << VW << ";\n";
+        for (auto &cv : cols) {
+            const int a = cv.first;
+            const Input &I = L.in[a];
+            Lay l{false, a};
+            const int cmin = cv.second.first, cmax = cv.second.second;
+            o << "      if (qq < " << FF.nq << " && fy >= " << -I.ey0 << " && fy < TY + " << I.ey1 << " && fx >= "
+              << -I.bx0 << " && fx + " << VW << " <= " << -I.bx0 + L.in_rw[a] << ") {\n";
+            o << "        const int fi = (fy - (" << ly0(l) << ")) * " << lw(l) << " + (fx - (" << lx0(l) << "));\n";
+            auto vload = [&](int cc, const std::string &dst_idx) {
+                // one vector of the unit's VW lanes at plane offset cc; planes below the
+                // input's first loaded plane are never consumed: do not touch their slots
+                o << "          { const T2 v = (k + (" << cc << ") >= (" << I.qlo
+                  << ")) ? *reinterpret_cast<const T2 *>(" << bname(l, cc) << " + fi) : T2{};\n";
+                const char *comp[4] = {"x", "y", "z", "w"};
+                for (int e2 = 0; e2 < VW; ++e2)
+                    o << "            " << gqname(PosKey{false, a, 0, e2, 0}) << "[b][" << dst_idx << "] = v."
+                      << comp[e2] << ";\n";
+                o << "          }\n";
+            };
+            o << "        if (k == KF) {\n";
+            for (int cc = cmin; cc <= cmax; ++cc) vload(cc, num(cc - cmin));
+            o << "        } else {\n";
+            for (int e2 = 0; e2 < VW; ++e2) {
+                const std::string q = gqname(PosKey{false, a, 0, e2, 0});
+                for (int d = 0; d < cmax - cmin; ++d)
+                    o << "          " << q << "[b][" << d << "] = " << q << "[b][" << d + 1 << "];\n";
+            }
+            vload(cmax, num(cmax - cmin));
+            o << "        }\n      }\n";
+        }
+        o << "    }\n";
+    } else if (!gq.empty()) {
         auto gaddr = [&](const PosKey &k, int cc) {
             Lay l{false, k.id};
             return bname(l, cc) + " + cb_" + lname(l) + " + b * (YT * VY * " + num(lw(l)) + ") + (" +
@@ -724,8 +827,8 @@ std::string generate_launch(const stencil_program *p, Launch &L, int index, bool
           << (G.stored ? ", stored" : "") << (G.keep == Keep::Reg ? ", register" : ", smem ring")
           << " depth " << G.depth << "\n";
         // register-stage queues advance every step
-        if (G.keep == Keep::Reg && G.depth > 1) {
-            o << "      #pragma unroll\n      for (int b = 0; b < " << (FR ? num(frame_geo(L, G, VW).nb) : "CBY")
+        if (has_rq(L, G) && G.depth > 1) {
+            o << "      #pragma unroll\n      for (int b = 0; b < " << (FR2 ? num(FF.nb) : FR ? num(frame_geo(L, G, VW).nb) : "CBY")
               << "; ++b)\n"
               << "      #pragma unroll\n      for (int i = 0; i < " << NPB << "; ++i)\n"
               << "      #pragma unroll\n      for (int d = 0; d < " << G.depth - 1 << "; ++d) rq" << m
@@ -803,15 +906,22 @@ std::string generate_launch(const stencil_program *p, Launch &L, int index, bool
         std::string GX0 = "X0 + xt * VX", GY0 = "Y0 + by", GOFF = "cg + b * (YT * VY * XP)";
         std::string blk_close = "        }\n";
         if (FR) {
-            const FrameGeo f = frame_geo(L, G, VW);
+            const FrameGeo fs = frame_geo(L, G, VW);
+            const FrameGeo f = FR2 ? FF : fs;  // enumeration: own region, or the launch frame
             o << "        #pragma unroll\n        for (int b = 0; b < " << f.nb << "; ++b) {\n";
             o << "          const int qq = tid + b * NT;\n";
-            if (f.nq % L.nt) {
-                o << "          if (qq < " << f.nq << ") {\n";
-                blk_close = "          }\n        }\n";
-            }
             o << "          const int fy = " << f.y_lo << " + qq / " << f.cs << ", fx = " << f.x_lo << " + (qq % "
               << f.cs << ") * " << VW << ";\n";
+            std::string act;
+            if (f.nq % L.nt) act = "qq < " + num(f.nq);
+            if (FR2 && (fs.y_lo != FF.y_lo || fs.rows != FF.rows || fs.x_lo != FF.x_lo || fs.cs != FF.cs))
+                act += std::string(act.empty() ? "" : " && ") + "fy >= " + num(fs.y_lo) + " && fy < " +
+                       num(fs.y_lo + fs.rows) + " && fx >= " + num(fs.x_lo) + " && fx < " +
+                       num(fs.x_lo + fs.cs * VW);
+            if (!act.empty()) {
+                o << "          if (" << act << ") {\n";
+                blk_close = "          }\n        }\n";
+            }
             std::set<Lay> used;
             if (G.keep == Keep::Smem) used.insert(Lay{true, m});
             for (auto &kv : pos) used.insert(Lay{kv.first.stage, kv.first.id});
@@ -867,7 +977,7 @@ std::string generate_launch(const stencil_program *p, Launch &L, int index, bool
         }
         // expressions of the VX*VY block points
         auto core_operand = [&](const Src &s, int iy, int jx) -> std::string {
-            if (s.stage && L.st[s.idx].keep == Keep::Reg) {
+            if (s.stage && (L.st[s.idx].keep == Keep::Reg || (FR2 && s.dx == 0 && s.dy == 0))) {
                 const Stage &P = L.st[s.idx];
                 int d = G.lead + s.dz - P.lead + P.depth - 1;
                 return "rq" + num(s.idx) + "[b][" + num(iy * VX + jx) + "][" + num(d) + "]";
@@ -982,7 +1092,8 @@ std::string generate_launch(const stencil_program *p, Launch &L, int index, bool
                         o << "          *(" << a << " + " << jx << ") = o" << iy << "_" << jx << ";\n";
                 }
             }
-        } else {
+        }
+        if (has_rq(L, G)) {
             for (int iy = 0; iy < VY; ++iy)
                 for (int jx = 0; jx < VX; ++jx)
                     o << "          rq" << m << "[b][" << iy * VX + jx << "][" << G.depth - 1 << "] = o"

@@ -389,7 +389,9 @@ void choose_config(const stencil_program *p, Launch &L, bool quick) {
     const int e = p->elem;
     const int64_t nz = g.nz_local;
     const Options &o = p->opt;
-    L.fr = frame_eligible(p, L) && (L.frame_pin >= 0 ? L.frame_pin != 0 : o.frame != 0);
+    const int fmode = L.frame_pin >= 0 ? L.frame_pin : o.frame;
+    L.fr = frame_eligible(p, L) && fmode != 0;
+    L.fr2 = L.fr && fmode == 2;
     const bool fr = L.fr;
     const int VW = 16 / e;
     std::vector<int> cx, cz, cn, cp, cvx, cvy, ccb, cty;
@@ -445,7 +447,7 @@ void choose_config(const stencil_program *p, Launch &L, bool quick) {
                                 Launch C = L;
                                 C.tx = tx; C.ty = ty; C.zc = (int)std::min<int64_t>(zc, nz);
                                 C.pf = pf; C.nt = nt; C.vx = vx; C.vy = fr ? 1 : vy; C.cby = cby;
-                                C.zq = fr ? 0 : o.zqueue;
+                                C.zq = fr ? (L.fr2 ? 2 : 0) : o.zqueue;
                                 C.nth = nt + (o.loader == 0 ? 32 : 0);
                                 layout_launch(p, C);
                                 if (C.smem > 227 * 1024) continue;
@@ -506,6 +508,14 @@ void choose_config(const stencil_program *p, Launch &L, bool quick) {
                     }
             }
         }
+    }
+    if (best_t >= 1e299 && L.fr2) {
+        // frame mode 2's register queues do not fit at any shape: plain frame mode
+        Launch R = L;
+        R.frame_pin = 1;
+        choose_config(p, R, quick);
+        L = R;
+        return;
     }
     if (best_t >= 1e299)
         fail(SP_E_RESOURCES, "group '" + L.name + "': no tile configuration fits in 227 KB of "

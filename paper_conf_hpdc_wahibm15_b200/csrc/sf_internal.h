@@ -149,6 +149,7 @@ struct Launch {
     int fastpath = -1;       // per-launch pin of the "fastpath" codegen variant (-1: option)
     int frame_pin = -1;      // per-launch pin of the "frame" evaluation mode (-1: option)
     bool fr = false;         // region-vector evaluation (resolved from pin/option/eligibility)
+    bool fr2 = false;        // frame mode with position-stable units and register z-reuse
 };
 
 struct Mode {

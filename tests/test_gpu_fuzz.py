@@ -16,7 +16,7 @@ from _harness import assert_close, gpu_run, oracle_outputs
 pytestmark = pytest.mark.gpu
 
 
-@pytest.mark.parametrize("frame", [0, 1], ids=["block", "frame"])
+@pytest.mark.parametrize("frame", [0, 1, 2], ids=["block", "frame", "frame2"])
 @pytest.mark.parametrize("boxes", [False, True], ids=["full", "boxed"])
 @pytest.mark.parametrize("seed", range(12))
 def test_fuzz_parity_bitexact(cuda_device, seed, boxes, frame):

@@ -369,16 +369,18 @@ FRAME_TILES = [{}, dict(tile_x=16, tile_y=3, zchunk=2, threads=32),
                dict(tile_x=32, tile_y=4, zchunk=9, threads=64, fastpath=1)]
 
 
+@pytest.mark.parametrize("frame", [1, 2])
 @pytest.mark.parametrize("name,prog,plans", CASES, ids=[c[0] for c in CASES])
 @pytest.mark.parametrize("fmad", [0, 1])
-def test_frame_mode_parity(cuda_device, name, prog, plans, fmad):
-    """frame=1: fused plans (complex fusion with halo recompute, fission+fusion) match
+def test_frame_mode_parity(cuda_device, name, prog, plans, fmad, frame):
+    """frame=1 / 2 (2: one unit grid per launch, own-position taps from register
+    queues): fused plans (complex fusion with halo recompute, fission+fusion) match
     the oracle bit-exactly in the parity build and within R17 in the perf build."""
     ref = oracle_outputs(prog, seed=12)
     for tiles in FRAME_TILES:
         for plan in plans:
             try:
-                got = gpu_run(prog, "fused", 12, options=dict(tiles, fmad=fmad, frame=1),
+                got = gpu_run(prog, "fused", 12, options=dict(tiles, fmad=fmad, frame=frame),
                               plan=prog["plans"][plan])
             except StencilError as e:  # a pinned tile whose rings exceed shared memory
                 assert tiles and e.code == 6, e
@@ -391,5 +393,7 @@ def test_frame_mode_c4_reduced_bitexact(cuda_device):
     prog = _c4_small()
     ref = oracle_outputs(prog, seed=13)
     for tiles in ({}, dict(tile_x=32, tile_y=5, zchunk=4, threads=64)):
-        got = gpu_run(prog, "fused", 13, options=dict(tiles, fmad=0, frame=1), plan=prog["plans"]["fused"])
-        assert_close(prog, got, ref, exact=True)
+        for frame in (1, 2):
+            got = gpu_run(prog, "fused", 13, options=dict(tiles, fmad=0, frame=frame),
+                          plan=prog["plans"]["fused"])
+            assert_close(prog, got, ref, exact=True)

@@ -42,17 +42,18 @@ def main():
     ap.add_argument("--wide", action="store_true")
     ap.add_argument("--iters", type=int, default=5)
     ap.add_argument("--out")
+    ap.add_argument("--plan-file", help="groups from a plan file (\"groups\") instead of the named plan")
     a = ap.parse_args()
     opts = {kv.split("=")[0]: int(kv.split("=")[1]) for kv in a.opt}
     prog = bench.load_workload(a.workload)
-    plan = bench.plan_of(prog, a.plan)
+    plan = json.load(open(a.plan_file))["groups"] if a.plan_file else bench.plan_of(prog, a.plan)
     dev = torch.device("cuda:0")
     base = Program(prog, options=opts)
     base.set_plan(plan)
     base.allocate(dev, fill=0.0)
     bench.fill_inputs(base, prog, dev, 0, prog["grid"]["ghost"][2])
     n = base.n_launches("fused")
-    cands = list(candidates(prog["dtype"], a.wide))
+    cands = [{}] + list(candidates(prog["dtype"], a.wide))  # {}: the model-driven chooser
 
     def build(c):
         p = Program(prog, options=opts)

@@ -41,7 +41,13 @@ def single(seed, boxes, frame=False):
     ref = oracle_outputs(prog, seed=seed, poison=False)
     tiles = FRAME_TILES if frame else TILES
     opts = dict(tiles[int(rng.integers(0, len(tiles)))], fmad=0)
-    assert_close(prog, gpu_run(prog, "unfused", seed, options=opts, poison=False), ref, exact=True)
+    if frame:
+        opts["frame"] = frame
+        if boxes:  # loop-bounded groups keep the block form: no frame-only (free tile_y) shapes
+            opts = {"fmad": 0, "frame": frame}
+    # frame shapes (free tile_y) apply to fused groups; the unfused kernels keep the block form
+    uopts = {"fmad": 0} if frame else opts
+    assert_close(prog, gpu_run(prog, "unfused", seed, options=uopts, poison=False), ref, exact=True)
     for plan in plans:
         got = gpu_run(prog, "fused", seed, options=opts, plan=plan, poison=False)
         assert_close(prog, got, ref, exact=True)
@@ -126,7 +132,7 @@ def main():
     ap.add_argument("--seeds", type=int, default=200)
     ap.add_argument("--start", type=int, default=1000)
     ap.add_argument("--ranks", type=int, default=0)
-    ap.add_argument("--frame", action="store_true", help="fused plans in region-vector (frame) mode")
+    ap.add_argument("--frame", type=int, default=0, help="fused plans in region-vector (frame) mode 1 / 2")
     a = ap.parse_args()
     fails = 0
     for seed in range(a.start, a.start + a.seeds):

@@ -648,3 +648,20 @@ def test_frame_mode_codegen_and_pins(name):
     # and the pin can switch it off again for that launch only
     p.tune("fused", 0, dict(frame=0))
     assert "_f[i]" in p.source("fused")
+
+
+def test_frame2_queues_and_fallback():
+    """frame=2: one unit grid per launch with register queues for own-position taps
+    (input queues "zg_", stage queues "rq" beside the shared-memory rings); a shape whose
+    queues cannot fit in 255 registers falls back to frame mode 1 instead of failing."""
+    prog = P.c3(n=64)
+    p = Program(prog, options={"frame": 2})
+    p.set_plan(prog["plans"]["fission_fused"])
+    g0 = p.source("fused").split("sf_fused_1")[0]
+    assert "zg_I" in g0 and "rq0[" in g0 and "fi_" in g0
+    p.tune("fused", 0, dict(tile_x=64, tile_y=16, threads=32, zchunk=8, frame=2))
+    r = p.report("fused", 0)
+    g0 = p.source("fused").split("sf_fused_1")[0]
+    assert (r["tile_x"], r["tile_y"], r["threads"]) == (64, 16, 32)
+    assert "fi_" in g0 and "zg_I" not in g0      # frame mode 1 at that shape
+    p.compile("fused")

@@ -234,6 +234,8 @@ sp_status stencil_program_bind(stencil_program *prog, int32_t array, void *dev_p
  *   "fastpath"  1: a second, predicate-free copy of the step body for interior
  *               tiles/planes (fewer issued instructions, larger code); default 0
  *   "minblocks" __launch_bounds__ minimum resident CTAs (ptxas register budget)
+ *   "psleep"    ns: the TMA producer warp waits for a free ring slot with nanosleep
+ *               back-off starting at this value (default 32; 0 = spin on try_wait)
  *   "frame"     1: region-vector evaluation of fused launches: every statement is
  *               evaluated on its whole extended region (tile + halo of complex
  *               fusion, §5.5.3) in 16-byte x-vectors of adjacent points

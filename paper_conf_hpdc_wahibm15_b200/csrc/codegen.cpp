@@ -473,8 +473,12 @@ std::string generate_launch(const stencil_program *p, Launch &L, int index, bool
         o << "      for (int j = KF; j < zc; ++j) {\n";
         if (L2PF > 0) l2_prefetch("(j + " + num(L2PF) + ")", "        ");
         o << "        const int s = j - 1 - PF;  // step whose slots batch j overwrites\n";
-        o << "        if (s >= KF) sf_mbar_wait(&empty[(s - KF) & " << NE - 1 << "], ((s - KF) >> "
-          << log2i(NE) << ") & 1);\n";
+        if (p->opt.psleep > 0)
+            o << "        if (s >= KF) sf_mbar_wait_backoff(&empty[(s - KF) & " << NE - 1 << "], ((s - KF) >> "
+              << log2i(NE) << ") & 1, " << p->opt.psleep << "u);\n";
+        else
+            o << "        if (s >= KF) sf_mbar_wait(&empty[(s - KF) & " << NE - 1 << "], ((s - KF) >> "
+              << log2i(NE) << ") & 1);\n";
         batch(o, "        ");
         o << "      }\n    }\n";
         if (CX > 1) o << "    sf_cluster_sync();  // no CTA leaves while a neighbour may read its rings\n";

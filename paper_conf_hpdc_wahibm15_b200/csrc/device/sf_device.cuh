@@ -65,6 +65,24 @@ __device__ __forceinline__ void sf_mbar_wait(sf_u64 *bar, sf_u32 parity) {
 #endif
 }
 
+// Producer-side wait for a free ring slot with exponential nanosleep back-off (start
+// `ns`, capped at 8x): the producer warp is idle most of the time, and a tight try_wait
+// loop spends issue slots of its SM sub-partition (and power) the compute warps need;
+// the slot is needed only PF steps later, so a sleeping producer costs no latency.
+__device__ __forceinline__ void sf_mbar_wait_backoff(sf_u64 *bar, sf_u32 parity, unsigned ns) {
+    unsigned t = ns;
+    for (;;) {
+        sf_u32 done;
+        asm volatile(
+            "{\n\t.reg .pred P1;\n\t"
+            "mbarrier.try_wait.parity.shared::cta.b64 P1, [%1], %2;\n\t"
+            "selp.u32 %0, 1, 0, P1;\n}" : "=r"(done) : "r"(sf_smem_addr(bar)), "r"(parity) : "memory");
+        if (done) return;
+        __nanosleep(t);
+        t = t < 8 * ns ? 2 * t : t;
+    }
+}
+
 // consumer release of a ring slot (default .release.cta semantics)
 __device__ __forceinline__ void sf_mbar_arrive(sf_u64 *bar) {
     asm volatile("mbarrier.arrive.shared::cta.b64 _, [%0];" ::"r"(sf_smem_addr(bar)) : "memory");

@@ -54,6 +54,9 @@ struct Options {
     int minblocks = 1; // __launch_bounds__ minimum resident CTAs (register budget for ptxas)
     int cluster_x = 1; // > 1: CTAs per cluster along x sharing x-halos of smem stages over DSMEM
     int frame = 0;     // region-vector evaluation of fused launches (see stencilfuse.h "frame")
+    int psleep = 32;   // producer waits for a free ring slot with nanosleep back-off (ns; 0 = spin):
+                       // r2: the spinning producer warp issued 28 % of sf_fused_5's instructions;
+                       // 32 ns back-off: C4 -3.6 %, C3 -1.2 %, C2 -0.7 % (interleaved A/B)
     int halo_sel = 0;  // halo points: expression always evaluated, ghost value selected after
                        // (no branch around the loads: several halo points' loads interleave)
     int regcap = 1; // recompile a few registers tighter when that adds a resident CTA:

@@ -451,7 +451,11 @@ std::string generate_launch(const stencil_program *p, Launch &L, int index, bool
     L.pdl = pdl;
     if (pdl) o << "  sf_pdl_launch_dependents();  // the next group may start its prologue\n";
     if (tma) {
-        o << "  if (tid >= NT) {  // ---- TMA producer warp: batch j for step j, PF steps ahead\n";
+        // the role test uses a warp-uniform value (a shuffle broadcast of the warp index): with
+        // a per-thread test ptxas treats the compute loop as possibly divergent and keeps
+        // uniform values (the step index, the coefficient-table loads) out of the uniform
+        // datapath (micro-kernels: LDC into general registers instead of LDCU)
+        o << "  if (__shfl_sync(0xffffffffu, tid >> 5, 0) >= NT / 32) {  // ---- TMA producer warp: batch j for step j, PF steps ahead\n";
         o << "    if (tid == NT) {\n";
         if (pdl) o << "      sf_pdl_wait();  // inputs written by the previous group are complete\n";
         const int L2PF = p->opt.l2pf;
@@ -473,7 +477,10 @@ std::string generate_launch(const stencil_program *p, Launch &L, int index, bool
         o << "      for (int j = KF; j < zc; ++j) {\n";
         if (L2PF > 0) l2_prefetch("(j + " + num(L2PF) + ")", "        ");
         o << "        const int s = j - 1 - PF;  // step whose slots batch j overwrites\n";
-        if (p->opt.psleep > 0)
+        if (p->opt.phint > 0)
+            o << "        if (s >= KF) sf_mbar_wait_hint(&empty[(s - KF) & " << NE - 1 << "], ((s - KF) >> "
+              << log2i(NE) << ") & 1, " << p->opt.phint << "u);\n";
+        else if (p->opt.psleep > 0)
             o << "        if (s >= KF) sf_mbar_wait_backoff(&empty[(s - KF) & " << NE - 1 << "], ((s - KF) >> "
               << log2i(NE) << ") & 1, " << p->opt.psleep << "u);\n";
         else
@@ -653,8 +660,12 @@ std::string generate_launch(const stencil_program *p, Launch &L, int index, bool
 
     // ------------------------------------------------------------- z-march
     for (int r = 0; r < n_ready; ++r) o << "  unsigned cph" << r << " = 0;\n";
+    // coef_const 2: a toggle used only to index the zero table keeps the coefficient address
+    // warp-uniform in ptxas's analysis (the step index itself feeds per-thread addressing and
+    // lives in a general register), so each coefficient is one LDCU into a uniform register
+    if (cc2) o << "  unsigned sfc = 0u;\n";
     o << "  for (int k = KF; k < zc; ++k) {\n";
-    if (cc2) o << "    const int sfz = SFZ[k & 1];  // always 0 (see coef_ref)\n";
+    if (cc2) o << "    sfc ^= 1u;\n    const int sfz = SFZ[sfc];  // always 0 (see coef_ref)\n";
     if (tma) {
         o << "    sf_mbar_wait(&full[(k - KF) & " << NB - 1 << "], ((k - KF) >> " << log2i(NB)
           << ") & 1);\n";

@@ -83,6 +83,20 @@ __device__ __forceinline__ void sf_mbar_wait_backoff(sf_u64 *bar, sf_u32 parity,
     }
 }
 
+// Producer-side wait with a suspend-time hint: try_wait suspends the thread until the phase
+// completes or the hint (ns) elapses, so the idle producer issues a handful of instructions per
+// step instead of a polling loop (the hint is not used for the compute warps' waits: there a
+// late wake-up is on the critical path).
+__device__ __forceinline__ void sf_mbar_wait_hint(sf_u64 *bar, sf_u32 parity, sf_u32 ns) {
+    asm volatile(
+        "{\n\t.reg .pred P1;\n"
+        "SF_WAITH_%=:\n\t"
+        "mbarrier.try_wait.parity.shared::cta.b64 P1, [%0], %1, %2;\n\t"
+        "@!P1 bra SF_WAITH_%=;\n}" ::"r"(sf_smem_addr(bar)),
+        "r"(parity), "r"(ns)
+        : "memory");
+}
+
 // consumer release of a ring slot (default .release.cta semantics)
 __device__ __forceinline__ void sf_mbar_arrive(sf_u64 *bar) {
     asm volatile("mbarrier.arrive.shared::cta.b64 _, [%0];" ::"r"(sf_smem_addr(bar)) : "memory");

@@ -54,6 +54,7 @@ struct Options {
     int minblocks = 1; // __launch_bounds__ minimum resident CTAs (register budget for ptxas)
     int cluster_x = 1; // > 1: CTAs per cluster along x sharing x-halos of smem stages over DSMEM
     int frame = 0;     // region-vector evaluation of fused launches (see stencilfuse.h "frame")
+    int phint = 0;     // > 0: producer waits with try_wait suspend-time hint (ns) instead of psleep
     int psleep = 32;   // producer waits for a free ring slot with nanosleep back-off (ns; 0 = spin):
                        // r2: the spinning producer warp issued 28 % of sf_fused_5's instructions;
                        // 32 ns back-off: C4 -3.6 %, C3 -1.2 %, C2 -0.7 % (interleaved A/B)

@@ -665,3 +665,18 @@ def test_frame2_queues_and_fallback():
     assert (r["tile_x"], r["tile_y"], r["threads"]) == (64, 16, 32)
     assert "fi_" in g0 and "zg_I" not in g0      # frame mode 1 at that shape
     p.compile("fused")
+
+
+def test_producer_wait_variants_codegen():
+    """The TMA producer waits for a free ring slot with nanosleep back-off by default
+    (option psleep, ns), spins with psleep=0, or uses a try_wait suspend hint (phint);
+    the role test is warp-uniform (shuffle broadcast of the warp index)."""
+    prog = P.c2(n=64)
+    for opts, want in (({}, "sf_mbar_wait_backoff(&empty"), ({"psleep": 0}, "sf_mbar_wait(&empty"),
+                       ({"phint": 5000}, "sf_mbar_wait_hint(&empty")):
+        p = Program(prog, options=opts)
+        p.set_plan(prog["plans"]["fused"])
+        src = p.source("fused")
+        assert want in src, opts
+        assert "__shfl_sync(0xffffffffu, tid >> 5, 0) >= NT / 32" in src
+    p.compile("fused")

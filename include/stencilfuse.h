@@ -236,6 +236,7 @@ sp_status stencil_program_bind(stencil_program *prog, int32_t array, void *dev_p
  *   "minblocks" __launch_bounds__ minimum resident CTAs (ptxas register budget)
  *   "psleep"    ns: the TMA producer warp waits for a free ring slot with nanosleep
  *               back-off starting at this value (default 32; 0 = spin on try_wait)
+ *   "phint", "pbar", "pow2ring"   measured-off producer-wait / ring experiments
  *   "frame"     1: region-vector evaluation of fused launches: every statement is
  *               evaluated on its whole extended region (tile + halo of complex
  *               fusion, §5.5.3) in 16-byte x-vectors of adjacent points

@@ -426,6 +426,8 @@ sp_status sp_program_set_option(stencil_program *p, const char *key, int64_t v) 
         else if (k == "frame") o.frame = (int)std::min<int64_t>(v, 2);
         else if (k == "psleep") o.psleep = (int)std::min<int64_t>(v, 10000);
         else if (k == "phint") o.phint = (int)std::min<int64_t>(v, 1000000);
+        else if (k == "pow2ring") o.pow2ring = v != 0;
+        else if (k == "pbar") o.pbar = v != 0;
         else if (k == "l2_flush") {}
         else fail(SP_E_ARG, "unknown option '" + k + "'");
         if (v < 0 && k != "prefetch") fail(SP_E_ARG, "negative option value");

@@ -456,7 +456,12 @@ std::string generate_launch(const stencil_program *p, Launch &L, int index, bool
         // uniform values (the step index, the coefficient-table loads) out of the uniform
         // datapath (micro-kernels: LDC into general registers instead of LDCU)
         o << "  if (__shfl_sync(0xffffffffu, tid >> 5, 0) >= NT / 32) {  // ---- TMA producer warp: batch j for step j, PF steps ahead\n";
-        o << "    if (tid == NT) {\n";
+        // pbar: the whole producer warp runs the loop and blocks in bar.sync on the step's
+        // named barrier until every compute warp has arrived (hardware wait, no polling); one
+        // elected lane issues the TMA work.  Named barrier ids 2 .. 2+NE-1 (id 1: compute sync)
+        const bool PB = p->opt.pbar && CX == 1 && !L.xp && NE <= 8;
+        L.pbar = PB;
+        o << (PB ? "    const bool lead = tid == NT;\n    {\n" : "    if (tid == NT) {\n");
         if (pdl) o << "      sf_pdl_wait();  // inputs written by the previous group are complete\n";
         const int L2PF = p->opt.l2pf;
         auto l2_prefetch = [&](const std::string &jexpr, const std::string &ind) {
@@ -470,14 +475,20 @@ std::string generate_launch(const stencil_program *p, Launch &L, int index, bool
             }
         };
         if (L2PF > 0) {
-            o << "      for (int j = KF + 1; j < min(KF + " << L2PF << ", zc); ++j) {\n";
+            o << "      " << (PB ? "if (lead) " : "") << "for (int j = KF + 1; j < min(KF + " << L2PF << ", zc); ++j) {\n";
             l2_prefetch("j", "        ");
             o << "      }\n";
         }
         o << "      for (int j = KF; j < zc; ++j) {\n";
-        if (L2PF > 0) l2_prefetch("(j + " + num(L2PF) + ")", "        ");
+        if (L2PF > 0) {
+            if (PB) o << "        if (lead) {\n";
+            l2_prefetch("(j + " + num(L2PF) + ")", "        ");
+            if (PB) o << "        }\n";
+        }
         o << "        const int s = j - 1 - PF;  // step whose slots batch j overwrites\n";
-        if (p->opt.phint > 0)
+        if (PB)
+            o << "        if (s >= KF) sf_bar_sync(2 + ((s - KF) & " << NE - 1 << "), NT + 32);\n";
+        else if (p->opt.phint > 0)
             o << "        if (s >= KF) sf_mbar_wait_hint(&empty[(s - KF) & " << NE - 1 << "], ((s - KF) >> "
               << log2i(NE) << ") & 1, " << p->opt.phint << "u);\n";
         else if (p->opt.psleep > 0)
@@ -486,8 +497,14 @@ std::string generate_launch(const stencil_program *p, Launch &L, int index, bool
         else
             o << "        if (s >= KF) sf_mbar_wait(&empty[(s - KF) & " << NE - 1 << "], ((s - KF) >> "
               << log2i(NE) << ") & 1);\n";
+        if (PB) o << "        if (lead) {\n";
         batch(o, "        ");
-        o << "      }\n    }\n";
+        if (PB) o << "        }\n";
+        o << "      }\n";
+        if (PB)  // the last steps' barrier generations: the compute warps arrive on every step
+            o << "      for (int s = max(KF, zc - 1 - PF); s < zc; ++s) sf_bar_sync(2 + ((s - KF) & " << NE - 1
+              << "), NT + 32);\n";
+        o << "    }\n";
         if (CX > 1) o << "    sf_cluster_sync();  // no CTA leaves while a neighbour may read its rings\n";
         o << "    return;\n  }\n";
     }
@@ -1254,8 +1271,12 @@ std::string generate_launch(const stencil_program *p, Launch &L, int index, bool
         emit_body(false);
     }
     if (tma) {
-        o << "    __syncwarp();\n";
-        o << "    if ((tid & 31) == 0) sf_mbar_arrive(&empty[(k - KF) & " << NE - 1 << "]);\n";
+        if (L.pbar) {
+            o << "    sf_bar_arrive(2 + ((k - KF) & " << NE - 1 << "), NT + 32);  // slots of step k are free\n";
+        } else {
+            o << "    __syncwarp();\n";
+            o << "    if ((tid & 31) == 0) sf_mbar_arrive(&empty[(k - KF) & " << NE - 1 << "]);\n";
+        }
     } else {
         o << "    sf_bar_sync(1, NT);\n";
     }

@@ -103,6 +103,11 @@ __device__ __forceinline__ void sf_mbar_arrive(sf_u64 *bar) {
 }
 
 // named barrier over the compute warps only (the producer warp never joins)
+// named-barrier arrive (no wait): the compute warps' "slot free" signal to a producer
+// warp blocked in bar.sync on the same id (option pbar)
+__device__ __forceinline__ void sf_bar_arrive(int id, int nthreads) {
+    asm volatile("bar.arrive %0, %1;" ::"r"(id), "r"(nthreads) : "memory");
+}
 __device__ __forceinline__ void sf_bar_sync(int id, int nthreads) {
     asm volatile("bar.sync %0, %1;" ::"r"(id), "r"(nthreads) : "memory");
 }

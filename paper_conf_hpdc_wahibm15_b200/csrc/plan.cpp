@@ -255,6 +255,7 @@ static void layout_launch(const stencil_program *p, Launch &L) {
         // reads of edge lanes past a row end, so they never touch a slot being refilled
         int64_t plane = rup((int64_t)rw * rh, 128 / e) + (L.fr ? 128 / e : 0);
         int D = I.ahi - I.alo + 1 + L.pf;  // ring slot = plane mod D (constant modulo per step)
+        if (p->opt.pow2ring) D = pow2ceil(D);  // slot = a mask instead of a multiply-high modulo
         L.in_off.push_back(off);
         L.in_plane.push_back(plane);
         L.in_rw.push_back(rw);
@@ -273,6 +274,7 @@ static void layout_launch(const stencil_program *p, Launch &L) {
         if (G.keep == Keep::Smem) {
             // one plane deeper than the reuse distance: no end-of-step barrier needed
             int D = G.depth + 1;
+            if (p->opt.pow2ring) D = pow2ceil(D);
             int64_t plane = rup((int64_t)w * h, 128 / e) + (L.fr ? 128 / e : 0);
             L.st_off.push_back(off);
             L.st_plane.push_back(plane);

@@ -54,6 +54,8 @@ struct Options {
     int minblocks = 1; // __launch_bounds__ minimum resident CTAs (register budget for ptxas)
     int cluster_x = 1; // > 1: CTAs per cluster along x sharing x-halos of smem stages over DSMEM
     int frame = 0;     // region-vector evaluation of fused launches (see stencilfuse.h "frame")
+    int pbar = 0;      // 1: "slot free" via named barriers (producer blocks in bar.sync, no polling)
+    int pow2ring = 0;  // ring depths rounded up to powers of two (slot = mask, more shared memory)
     int phint = 0;     // > 0: producer waits with try_wait suspend-time hint (ns) instead of psleep
     int psleep = 32;   // producer waits for a free ring slot with nanosleep back-off (ns; 0 = spin):
                        // r2: the spinning producer warp issued 28 % of sf_fused_5's instructions;
@@ -154,6 +156,7 @@ struct Launch {
     int frame_pin = -1;      // per-launch pin of the "frame" evaluation mode (-1: option)
     bool fr = false;         // region-vector evaluation (resolved from pin/option/eligibility)
     bool fr2 = false;        // frame mode with position-stable units and register z-reuse
+    bool pbar = false;       // "slot free" signalled through named barriers (codegen)
 };
 
 struct Mode {

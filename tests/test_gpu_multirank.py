@@ -116,7 +116,12 @@ def test_virtual_ranks_bitexact(cuda_device, cfg, ranks, fmad):
                                                  ("C4", 4, "fused", {}), ("chain3box", 3, "fused", {}),
                                                  ("C4", 3, "fused", {"fastpath": 1}),
                                                  ("C5", 2, "fused", {"fastpath": 1}),
-                                                 ("C3", 3, "unfused", {"fastpath": 1})])
+                                                 ("C3", 3, "unfused", {"fastpath": 1}),
+                                                 ("C3", 2, "fused", {"frame": 1}),
+                                                 ("C3", 3, "fused", {"frame": 2}),
+                                                 ("C2", 2, "fused", {"frame": 1, "fastpath": 1}),
+                                                 ("C5", 2, "fused", {"frame": 2}),
+                                                 ("C4", 2, "fused", {"psleep": 0})])
 def test_loopback_ranks_run_bitexact(cuda_device, cfg, ranks, mode, opts):
     """The executor's own multi-rank path (run_fused / run_unfused with a communicator:
     exchange schedule, interior planes overlapped with the exchange on the comm stream,

@@ -25,6 +25,15 @@
 // groups on B200 (SMEM : HBM bandwidth is only ~5.5 : 1) — by the reuse factor.
 // Halo strips (the extra layers of complex fusion) are evaluated point-wise.
 //
+// Region-vector form (option / pin "frame"): instead of register blocks on the tile
+// plus point-wise halo strips, every statement is evaluated on its whole extended
+// region in units of one 16-byte x-vector, enumerated linearly over the threads
+// (unit q = tid + b*NT); the region's x-range is rounded out to the vector
+// alignment and the extra lanes compute values no valid point consumes (their reads
+// past a row end land in the 128-B guard after every ring plane).  "frame=2" gives all
+// statements of a launch one unit grid (the union of their regions), so a unit's
+// own-position taps come from per-thread register queues.
+//
 // Ghost points (reading R1): a point outside the global interior takes the
 // array's ghost value through a predicated load; tiles inside the interior skip
 // the test.

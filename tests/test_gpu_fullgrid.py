@@ -90,7 +90,10 @@ def _check(workload, plan):
         print(f"{workload}/{plan} {n}: {g.size} points, inf-norm rel err {e:.3e}")
 
 
-@pytest.mark.parametrize("plan", ["measured", "fission_fused", "fused", "single", "unfused"])
+# fission_fused / fused run in the region-vector (frame) form at their bench pins; the
+# *_block plans keep the register-block form at its round-1 pins
+@pytest.mark.parametrize("plan", ["measured", "fission_fused", "fused", "single", "unfused",
+                                  "fission_fused_block"])
 def test_c3_full_grid(cuda_device, plan):
     _check("C3", plan)
 

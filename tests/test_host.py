@@ -680,3 +680,26 @@ def test_producer_wait_variants_codegen():
         assert want in src, opts
         assert "__shfl_sync(0xffffffffu, tid >> 5, 0) >= NT / 32" in src
     p.compile("fused")
+
+
+def test_ring_and_barrier_options_codegen():
+    """pow2ring rounds every ring depth up to a power of two (more shared memory, a mask
+    slot); pbar signals "slot free" through named barriers (compute warps bar.arrive, the
+    whole producer warp bar.sync, ids 2..2+NE-1) instead of the empty mbarriers."""
+    prog = P.c3(n=64)
+    p = Program(prog)
+    p.set_plan(prog["plans"]["fission_fused"])
+    base = [r["smem_bytes"] for r in p.reports("fused")]
+    q = Program(prog, options={"pow2ring": 1})
+    q.set_plan(prog["plans"]["fission_fused"])
+    assert all(b2 >= b1 for b1, b2 in zip(base, [r["smem_bytes"] for r in q.reports("fused")]))
+    src = q.source("fused")
+    import re
+    depths = {int(d) for d in re.findall(r"% (\d+)u\) \*", src)}
+    assert depths and all(d & (d - 1) == 0 for d in depths), depths
+    b = Program(prog, options={"pbar": 1})
+    b.set_plan(prog["plans"]["fission_fused"])
+    src = b.source("fused")
+    assert "sf_bar_arrive(2 + ((k - KF)" in src and "sf_bar_sync(2 + ((s - KF)" in src
+    assert "sf_mbar_arrive(&empty" not in src
+    b.compile("fused")

@@ -231,7 +231,9 @@ sp_status stencil_program_bind(stencil_program *prog, int32_t array, void *dev_p
  *               without spills): 0 never, 1 peer-push kernels (default), 2 all
  *   "l2pf"      TMA L2 prefetch of input planes this many steps beyond the
  *               shared-memory ring (default 1; 0 off)
- *   "fastpath"  1: a second, predicate-free copy of the step body for interior
+ *   "fastpath"  2: as 1, and the fast body also runs each chunk's warm-up steps (only
+ *               chunks/tiles at the global boundary run the general body);
+ *               1: a second, predicate-free copy of the step body for interior
  *               tiles/planes (fewer issued instructions, larger code); default 0
  *   "minblocks" __launch_bounds__ minimum resident CTAs (ptxas register budget)
  *   "psleep"    ns: the TMA producer warp waits for a free ring slot with nanosleep
@@ -298,7 +300,8 @@ sp_status sp_plan_greedy(stencil_program *prog, int32_t cap, int32_t *n_groups,
 typedef struct {
     int32_t tile_x, tile_y, zchunk, threads, prefetch, block_x, block_y, block_cby;
     int32_t zqueue;
-    int32_t fastpath;  /* 0 = the program's "fastpath" option, 1 = off, 2 = on (this launch) */
+    int32_t fastpath;  /* 0 = the program's "fastpath" option, 1 = off, 2 = on, 3 = on incl.
+                          warm-up steps (this launch) */
     int32_t frame;     /* 0 = the program's "frame" option, 1 = off, 2 = on, 3 = on with
                           position-stable units and register z-reuse (this launch) */
 } sp_tile_config;

@@ -418,7 +418,7 @@ sp_status sp_program_set_option(stencil_program *p, const char *key, int64_t v) 
         else if (k == "zwave") o.zwave = (int)v;
         else if (k == "zwave_streams") o.zwave_streams = std::max(1, std::min(8, (int)v));
         else if (k == "xpush") o.xpush = v != 0;
-        else if (k == "fastpath") o.fastpath = v != 0;
+        else if (k == "fastpath") o.fastpath = (int)std::min<int64_t>(v, 2);
         else if (k == "cluster_x") o.cluster_x = (int)std::max<int64_t>(1, std::min<int64_t>(v, 8));
         else if (k == "minblocks") o.minblocks = (int)std::max<int64_t>(1, std::min<int64_t>(v, 32));
         else if (k == "regcap") o.regcap = (int)std::min<int64_t>(v, 2);

@@ -825,7 +825,13 @@ std::string generate_launch(const stencil_program *p, Launch &L, int index, bool
     bool any_boxed = false;
     for (const Stage &G : L.st)
         if (G.needed && p->stmts[G.gid].boxed) any_boxed = true;
-    const bool spec = (L.fastpath >= 0 ? L.fastpath : p->opt.fastpath) && !any_boxed;
+    const int fpmode = L.fastpath >= 0 ? L.fastpath : p->opt.fastpath;
+    const bool spec = fpmode != 0 && !any_boxed;
+    // fastpath 2: the fast body also runs the chunk's warm-up steps (statements before their
+    // first plane compute values nobody reads; stores keep a uniform plane-range test), so
+    // only chunks / tiles at the global boundary ever execute the general body — one hot
+    // body per CTA instead of two (the instruction cache held both, r2 measurements)
+    const bool spec2 = spec && fpmode == 2;
     if (spec) {
         int kst0 = INT32_MIN;
         int lmin = INT32_MAX, lmax = INT32_MIN, slmin = INT32_MAX, slmax = INT32_MIN;
@@ -837,9 +843,9 @@ std::string generate_launch(const stencil_program *p, Launch &L, int index, bool
             if (G.stored) { slmin = std::min(slmin, G.lead); slmax = std::max(slmax, G.lead); }
         }
         o << "    // fast-step window [sf_k0, sf_k1) of this chunk (see codegen.cpp)\n";
-        o << "    int sf_k0 = max(" << kst0 << ", ZLO - Z0 - (" << lmin << ")), sf_k1 = min(zc, ZHI - Z0 - ("
-          << lmax << "));\n";
-        if (slmin != INT32_MAX)
+        o << "    int sf_k0 = max(" << (spec2 ? std::string("KF") : num(kst0)) << ", ZLO - Z0 - (" << lmin
+          << ")), sf_k1 = min(zc, ZHI - Z0 - (" << lmax << "));\n";
+        if (slmin != INT32_MAX && !spec2)
             o << "    sf_k0 = max(sf_k0, -(" << slmin << ")); sf_k1 = min(sf_k1, zc - (" << slmax << "));\n";
     }
     auto emit_body = [&](const bool FP) {
@@ -930,7 +936,8 @@ std::string generate_launch(const stencil_program *p, Launch &L, int index, bool
             o << "        const bool zin = gz >= ZLO && gz < ZHI;\n";
         o << "        const bool zal = " << (FP ? "true" : "gz + OZA >= 0 && gz + OZA < ZA") << ";\n";
         o << "        T *const gpl = p.arr[" << L.arr_slot[G.out] << "] + (long long)(gz + OZA) * PLANE;\n";
-        if (G.stored) o << "        const bool zst = " << (FP ? "true" : "q >= 0 && q < zc") << ";\n";
+        if (G.stored)
+            o << "        const bool zst = " << (FP && !spec2 ? "true" : "q >= 0 && q < zc") << ";\n";
         if (FP)
             o << "        const bool fast = true;\n";
         else if (boxed)

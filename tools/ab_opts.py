@@ -1,6 +1,7 @@
 """Interleaved A/B of codegen option sets on one workload's fused step (dev tool).
 
 python tools/ab_opts.py C3 --plan fission_fused --rounds 5 'halo_sel=0' 'halo_sel=1'
+python tools/ab_opts.py C4 'psleep=32' 'pin_fastpath=2'      (pin_<k>: override every launch pin)
 
 Every option set gets its own Program over the SAME device arrays; rounds alternate
 the sets (drift on the box is +-5 %, larger than most single-option effects).  Prints
@@ -39,10 +40,16 @@ def main():
     plan = bench.plan_of(prog, a.plan)
     progs, base = [], None
     for spec in a.specs:
-        p = Program(prog, options=parse(spec))
+        # keys "pin_<k>" override <k> in every per-launch pin; the rest are program options
+        kv = parse(spec)
+        over = {k[4:]: v for k, v in kv.items() if k.startswith("pin_")}
+        p = Program(prog, options={k: v for k, v in kv.items() if not k.startswith("pin_")})
         p.set_plan(plan)
         if not a.no_tune:
             bench.apply_tuning(p, prog, a.plan)
+            if over:
+                for i, c in enumerate(bench.tuned_configs(prog, a.plan) or []):
+                    p.tune("fused", i, dict(c or {}, **over))
         if base is None:
             p.allocate(dev, fill=0.0)
             bench.fill_inputs(p, prog, dev, 0, prog["grid"]["ghost"][2])

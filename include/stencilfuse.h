@@ -236,6 +236,15 @@ sp_status stencil_program_bind(stencil_program *prog, int32_t array, void *dev_p
  *               1: a second, predicate-free copy of the step body for interior
  *               tiles/planes (fewer issued instructions, larger code); default 0
  *   "minblocks" __launch_bounds__ minimum resident CTAs (ptxas register budget)
+ *   "rename"    1 (default): in run_fused on one rank, every later group that stores a
+ *               TEMP array stores into its own instance (a library-allocated buffer of
+ *               the program layout; extra memory = sum over TEMPs of (writer groups - 1)
+ *               arrays), so TEMP reuse creates no WAR/WAW ordering between groups.  The
+ *               instances' ghost cells are copied from the bound TEMP buffer when it is
+ *               (re)bound: rebind a TEMP after changing its ghost cells.  0: off
+ *   "streams"   N (default 2): run_fused on one rank issues the launches along the group
+ *               dependency DAG (sp_plan_dag) on up to N streams forked from and joined
+ *               back into the caller's stream (events; graph-capturable); 1: in order
  *   "psleep"    ns: the TMA producer warp waits for a free ring slot with nanosleep
  *               back-off starting at this value (default 32; 0 = spin on try_wait)
  *   "phint", "pbar", "pow2ring"   measured-off producer-wait / ring experiments
@@ -430,6 +439,16 @@ sp_status sp_run_launch(stencil_program *prog, int32_t mode, int32_t launch, sp_
  * launch when its interior is empty); under "zwave" one per non-empty wave of
  * each launch.  NCCL's own kernels are not counted.  Host-only. */
 sp_status sp_run_launch_count(stencil_program *prog, int32_t mode, int32_t *n);
+
+/* Launch DAG of run_fused (mode 1) with options "rename" / "streams" (one rank): the
+ * earlier launches launch `launch` depends on — RAW / WAR / WAW on the buffer instance
+ * of an array (with "rename" every later writer group of a TEMP stores into its own
+ * instance, so TEMP reuse adds no WAR/WAW edge) — written to deps[0..min(cap, n)) with
+ * *n_deps = n, and the stream index it is issued on (0 = the caller's stream).  Without
+ * those options every launch depends on its predecessors through the arrays alone, and
+ * all run on stream 0.  Host-only; also valid for mode 0 (stream 0, plain edges). */
+sp_status sp_plan_dag(stencil_program *prog, int32_t mode, int32_t launch, int32_t cap, int32_t *deps,
+                      int32_t *n_deps, int32_t *stream);
 
 /* Exchange `depth` ghost planes of each listed array with the z-neighbours
  * (ncclSend/ncclRecv grouped; planes are contiguous, no packing).  Requires

@@ -440,6 +440,18 @@ class Program:
     def run(self, mode, stream=None):
         (self.run_fused if self._mode(mode) else self.run_unfused)(stream)
 
+    def dag(self, mode="fused"):
+        """[(dependencies, stream index)] per launch (sp_plan_dag): the launch DAG run_fused
+        follows with the options "rename" / "streams"."""
+        out = []
+        for i in range(self.n_launches(mode)):
+            buf = (ctypes.c_int32 * 64)()
+            nd, st = ctypes.c_int32(), ctypes.c_int32()
+            _check(lib().sp_plan_dag(self.handle, self._mode(mode), i, 64, buf, ctypes.byref(nd),
+                                     ctypes.byref(st)))
+            out.append((list(buf[:min(nd.value, 64)]), st.value))
+        return out
+
     def run_launch(self, mode, i, stream=None):
         _check(lib().sp_run_launch(self.handle, self._mode(mode), i, _stream_handle(stream)))
 

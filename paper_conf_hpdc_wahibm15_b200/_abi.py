@@ -101,7 +101,7 @@ EXPORTS = [
     "stencil_program_destroy", "stencil_program_layout", "stencil_program_bind",
     "sp_program_set_option", "sp_program_counts", "sp_program_edges", "sp_fission_components",
     "fusion_plan_set", "sp_plan_greedy", "sp_plan_search", "sp_plan_search_ex", "sp_plan_count", "sp_plan_report", "fusion_plan_report", "sp_plan_source",
-    "sp_plan_exchange", "sp_plan_wave_offsets", "sp_plan_tune", "sp_compile", "sp_load", "run_unfused", "run_fused", "sp_run_launch", "sp_run_launch_count", "exchange_halos", "sp_last_error",
+    "sp_plan_exchange", "sp_plan_wave_offsets", "sp_plan_tune", "sp_compile", "sp_load", "run_unfused", "run_fused", "sp_run_launch", "sp_run_launch_count", "sp_plan_dag", "exchange_halos", "sp_last_error",
 ]
 
 _lib = None
@@ -150,6 +150,7 @@ def lib():
             "run_fused": [vp, vp],
             "sp_run_launch": [vp, i32, i32, vp],
             "sp_run_launch_count": [vp, i32, P(i32)],
+            "sp_plan_dag": [vp, i32, i32, i32, P(i32), P(i32), P(i32)],
             "exchange_halos": [vp, i32, P(i32), i32, vp],
         }
         for name, args in sig.items():

@@ -222,12 +222,59 @@ static int count_launches(stencil_program *p, int mode) {
     return n;
 }
 
+// One rank, fused mode, options rename / streams: the launches follow the group DAG on up to
+// `streams` streams forked from (and joined back into) the caller's stream; a launch waits
+// on the events of its dependencies issued on other streams.  Graph-capturable.
+static void run_dag(stencil_program *p, Mode &m, void *stream) {
+    dag_analysis(p, m, true);
+    prepare_shadows(p, m, stream);  // before the fork: every stream sees initialised shadows
+    const int n = (int)m.launches.size();
+    int S = 1;
+    for (int s : m.stream_of) S = std::max(S, s + 1);
+    while ((int)p->dag_streams.size() < S - 1) {
+        cudaStream_t s;
+        if (cudaStreamCreateWithFlags(&s, cudaStreamNonBlocking) != cudaSuccess)
+            fail(SP_E_CUDA, "cudaStreamCreate");
+        p->dag_streams.push_back(s);
+    }
+    while ((int)p->dag_events.size() < n + S) {
+        cudaEvent_t ev;
+        if (cudaEventCreateWithFlags(&ev, cudaEventDisableTiming) != cudaSuccess)
+            fail(SP_E_CUDA, "cudaEventCreate");
+        p->dag_events.push_back(ev);
+    }
+    auto st = [&](int s) { return s == 0 ? (cudaStream_t)stream : (cudaStream_t)p->dag_streams[s - 1]; };
+    auto ev = [&](int k) { return (cudaEvent_t)p->dag_events[k]; };
+    if (S > 1) {  // fork
+        if (cudaEventRecord(ev(n), st(0)) != cudaSuccess) fail(SP_E_CUDA, "event record");
+        for (int s = 1; s < S; ++s)
+            if (cudaStreamWaitEvent(st(s), ev(n), 0) != cudaSuccess) fail(SP_E_CUDA, "stream wait");
+    }
+    for (int i = 0; i < n; ++i) {
+        const int s = m.stream_of[i];
+        for (int d : m.deps[i])
+            if (m.stream_of[d] != s && cudaStreamWaitEvent(st(s), ev(d), 0) != cudaSuccess)
+                fail(SP_E_CUDA, "stream wait");
+        launch(p, m, i, st(s));
+        if (S > 1 && cudaEventRecord(ev(i), st(s)) != cudaSuccess) fail(SP_E_CUDA, "event record");
+    }
+    for (int s = 1; s < S; ++s) {  // join
+        if (cudaEventRecord(ev(n + s), st(s)) != cudaSuccess ||
+            cudaStreamWaitEvent(st(0), ev(n + s), 0) != cudaSuccess)
+            fail(SP_E_CUDA, "event join");
+    }
+}
+
 static void run_mode(stencil_program *p, int mode, void *stream) {
     Mode &m = mode_of(p, mode);
     load_mode(p, m);
     const bool multi = p->comm && p->comm->nranks > 1;
     if (mode == 1 && p->opt.zwave > 0 && !multi) {
         run_waves(p, m, stream);
+        return;
+    }
+    if (!multi && mode == 1 && (p->opt.rename || p->opt.streams > 1)) {
+        run_dag(p, m, stream);
         return;
     }
     if (!multi) {
@@ -327,6 +374,10 @@ void stencil_program_destroy(stencil_program *p) {
         for (void *e : p->events) cudaEventDestroy((cudaEvent_t)e);
         for (void *e : p->wave_events) cudaEventDestroy((cudaEvent_t)e);
         for (void *s : p->wave_streams) cudaStreamDestroy((cudaStream_t)s);
+        for (void *e : p->dag_events) cudaEventDestroy((cudaEvent_t)e);
+        for (void *s : p->dag_streams) cudaStreamDestroy((cudaStream_t)s);
+        for (auto &v : p->shadow)
+            for (void *q : v) cudaFree(q);
         if (p->sig) cudaFree(p->sig);
     });
     delete p;
@@ -428,6 +479,8 @@ sp_status sp_program_set_option(stencil_program *p, const char *key, int64_t v) 
         else if (k == "phint") o.phint = (int)std::min<int64_t>(v, 1000000);
         else if (k == "pow2ring") o.pow2ring = v != 0;
         else if (k == "pbar") o.pbar = v != 0;
+        else if (k == "rename") o.rename = v != 0;
+        else if (k == "streams") o.streams = (int)std::max<int64_t>(1, std::min<int64_t>(v, 8));
         else if (k == "l2_flush") {}
         else fail(SP_E_ARG, "unknown option '" + k + "'");
         if (v < 0 && k != "prefetch") fail(SP_E_ARG, "negative option value");
@@ -667,6 +720,20 @@ sp_status sp_run_launch_count(stencil_program *p, int32_t mode, int32_t *n) {
     return guard([&] {
         if (!p || !n) fail(SP_E_ARG, "null argument");
         *n = count_launches(p, mode);
+    });
+}
+
+sp_status sp_plan_dag(stencil_program *p, int32_t mode, int32_t launch, int32_t cap, int32_t *deps,
+                      int32_t *n_deps, int32_t *stream) {
+    return guard([&] {
+        if (!p || !n_deps || !stream || (cap > 0 && !deps)) fail(SP_E_ARG, "null argument");
+        Mode &m = mode_of(p, mode);
+        if (launch < 0 || launch >= (int)m.launches.size()) fail(SP_E_ARG, "bad launch index");
+        dag_analysis(p, m, mode == 1);
+        const std::vector<int> &d = m.deps[launch];
+        for (int k = 0; k < std::min<int>(cap, (int)d.size()); ++k) deps[k] = d[k];
+        *n_deps = (int)d.size();
+        *stream = m.stream_of[launch];
     });
 }
 

@@ -12,6 +12,7 @@
 #include <nvrtc.h>
 #include <nvtx3/nvToolsExt.h>
 
+#include <algorithm>
 #include <atomic>
 #include <cstdio>
 #include <cstdlib>
@@ -301,8 +302,104 @@ void *signal_block(stencil_program *p) {
     return p->sig;
 }
 
+// TEMP instances (option rename): reads of array a in launch i use instance rd_inst[i][a],
+// its stores (and the stage's ghost loads: ghost cells are identical in every instance)
+// wr_inst[i][a]; instance 0 is the bound buffer
+void dag_analysis(stencil_program *p, Mode &m, bool fused) {
+    if (m.dag_ok) return;
+    const int n = (int)m.launches.size(), na = (int)p->arrays.size();
+    const bool multi = p->comm && p->comm->nranks > 1;
+    const bool ren = fused && p->opt.rename && !multi && p->opt.zwave == 0 && p->opt.loader == 0;
+    std::vector<bool> renamable(na, false);
+    if (ren) {
+        for (int a = 0; a < na; ++a) renamable[a] = p->arrays[a].role == SP_TEMP;
+        for (const Stmt &S : p->stmts)  // a boxed write keeps the previous values: same buffer
+            if (S.boxed) renamable[S.out] = false;
+    }
+    m.rd_inst.assign(n, std::vector<int>(na, 0));
+    m.wr_inst.assign(n, std::vector<int>(na, 0));
+    m.n_inst.assign(na, 0);
+    std::vector<int> cur(na, 0);
+    std::vector<bool> written(na, false);
+    std::vector<std::set<int>> rd(n), wr(n);  // HBM reads / stores per launch
+    for (int i = 0; i < n; ++i) {
+        const Launch &L = m.launches[i];
+        m.rd_inst[i] = cur;
+        if (!L.dead) {
+            for (const Input &I : L.in) rd[i].insert(I.arr);
+            for (const Stage &G : L.st) {
+                if (!G.needed) continue;
+                if (p->stmts[G.gid].boxed) rd[i].insert(G.out);  // previous values outside the box
+                if (G.stored) wr[i].insert(G.out);
+            }
+        }
+        for (int a : wr[i]) {
+            if (renamable[a] && written[a]) cur[a] = ++m.n_inst[a];
+            written[a] = true;
+        }
+        m.wr_inst[i] = cur;
+    }
+    // dependencies on (array, instance): RAW, WAR, WAW
+    m.deps.assign(n, {});
+    for (int i = 0; i < n; ++i)
+        for (int j = 0; j < i; ++j) {
+            bool dep = false;
+            for (int a : wr[j]) {
+                if (rd[i].count(a) && m.wr_inst[j][a] == m.rd_inst[i][a]) dep = true;
+                if (wr[i].count(a) && m.wr_inst[j][a] == m.wr_inst[i][a]) dep = true;
+            }
+            for (int a : rd[j])
+                if (wr[i].count(a) && m.rd_inst[j][a] == m.wr_inst[i][a]) dep = true;
+            if (dep) m.deps[i].push_back(j);
+        }
+    // streams: a launch follows its latest dependency's stream, else the least-loaded one
+    const int S = (fused && !multi && p->opt.zwave == 0) ? std::max(1, p->opt.streams) : 1;
+    m.stream_of.assign(n, 0);
+    std::vector<int> load(S, 0);
+    for (int i = 0; i < n; ++i) {
+        int s = 0;
+        if (!m.deps[i].empty()) s = m.stream_of[m.deps[i].back()];
+        else s = (int)(std::min_element(load.begin(), load.end()) - load.begin());
+        m.stream_of[i] = s;
+        load[s] += m.launches[i].dead ? 0 : 1;
+    }
+    m.dag_ok = true;
+}
+
+static void *inst_ptr(stencil_program *p, int a, int inst) {
+    if (inst == 0) return p->ptrs[a];
+    return p->shadow[a][inst - 1];
+}
+
+void prepare_shadows(stencil_program *p, Mode &m, void *stream) {
+    const int na = (int)p->arrays.size();
+    if ((int)p->shadow.size() < na) p->shadow.resize(na);
+    if ((int)m.shadow_src.size() < na) m.shadow_src.assign(na, nullptr);
+    for (int a = 0; a < na; ++a) {
+        const int k = m.n_inst.empty() ? 0 : m.n_inst[a];
+        if (!k) continue;
+        if (!p->ptrs[a]) fail(SP_E_STATE, "array '" + p->arrays[a].name + "' is not bound");
+        // only a TEMP whose bound buffer changed needs its shadows (re)initialised: rebinding
+        // other arrays every step (double-buffered inputs) costs nothing here
+        if (m.shadow_src[a] == p->ptrs[a] && (int)p->shadow[a].size() >= k) continue;
+        while ((int)p->shadow[a].size() < k) {
+            void *q = nullptr;
+            if (cudaMalloc(&q, (size_t)p->layout.bytes) != cudaSuccess)
+                fail(SP_E_CUDA, "shadow buffer of '" + p->arrays[a].name + "' (option rename)");
+            p->shadow[a].push_back(q);
+        }
+        // the ghost cells every instance must carry (reading R1): a copy of the bound buffer
+        for (int j = 0; j < k; ++j)
+            cuda_check(cudaMemcpyAsync(p->shadow[a][j], p->ptrs[a], (size_t)p->layout.bytes,
+                                       cudaMemcpyDeviceToDevice, (cudaStream_t)stream),
+                       "shadow init copy");
+        m.shadow_src[a] = p->ptrs[a];
+    }
+}
+
 static void build_params(stencil_program *p, Mode &m) {
     if (m.maps_version == p->bind_version) return;
+    const bool inst = m.dag_ok && !m.rd_inst.empty();
     const int e = p->elem;
     const sp_layout &lay = p->layout;
     for (size_t i = 0; i < m.launches.size(); ++i) {
@@ -312,7 +409,7 @@ static void build_params(stencil_program *p, Mode &m) {
         blk.assign(L.param_size / 64 + 1, Mode::Blk{});
         unsigned char *buf = blk[0].b;
         for (size_t a = 0; a < L.in.size(); ++a) {
-            void *ptr = p->ptrs[L.in[a].arr];
+            void *ptr = inst ? inst_ptr(p, L.in[a].arr, m.rd_inst[i][L.in[a].arr]) : p->ptrs[L.in[a].arr];
             if (!ptr) fail(SP_E_STATE, "array '" + p->arrays[L.in[a].arr].name + "' is not bound");
             CUtensorMap tm;
             cuuint64_t dims[3] = {(cuuint64_t)lay.x_pitch, (cuuint64_t)lay.y_alloc,
@@ -330,7 +427,7 @@ static void build_params(stencil_program *p, Mode &m) {
             std::memcpy(buf + 128 * a, &tm, 128);
         }
         for (size_t s = 0; s < L.slot_arr.size(); ++s) {
-            void *ptr = p->ptrs[L.slot_arr[s]];
+            void *ptr = inst ? inst_ptr(p, L.slot_arr[s], m.wr_inst[i][L.slot_arr[s]]) : p->ptrs[L.slot_arr[s]];
             if (!ptr) fail(SP_E_STATE, "array '" + p->arrays[L.slot_arr[s]].name + "' is not bound");
             std::memcpy(buf + L.ptr_off + 8 * s, &ptr, 8);
         }
@@ -378,6 +475,8 @@ void launch(stencil_program *p, Mode &m, int i, void *stream, int z0, int z1, in
     const int n_hi = z3 > z2 ? (z3 - z2 + L.zc - 1) / L.zc : 0;
     const int nchunks = n_lo + n_hi;
     if (nchunks <= 0) return;
+    if (&m == &p->fused && (p->opt.rename || p->opt.streams > 1)) dag_analysis(p, m, true);
+    if (m.dag_ok && !m.n_inst.empty()) prepare_shadows(p, m, stream);
     build_params(p, m);
     // NVTX range per group launch (SURVEY.md §5 tracing): a tool (Nsight Systems) projects
     // it onto the kernel; a no-op without one attached

@@ -54,6 +54,10 @@ struct Options {
     int minblocks = 1; // __launch_bounds__ minimum resident CTAs (register budget for ptxas)
     int cluster_x = 1; // > 1: CTAs per cluster along x sharing x-halos of smem stages over DSMEM
     int frame = 0;     // region-vector evaluation of fused launches (see stencilfuse.h "frame")
+    int rename = 1;    // fused mode, one rank: every later writer group of a TEMP gets its own
+                       // buffer instance (no WAR/WAW through TEMP reuse between groups)
+    int streams = 2;   // fused mode, one rank: launches on up to this many streams along the
+                       // group dependency DAG (events between streams); r2: C4 -8.3 %
     int pbar = 0;      // 1: "slot free" via named barriers (producer blocks in bar.sync, no polling)
     int pow2ring = 0;  // ring depths rounded up to powers of two (slot = mask, more shared memory)
     int phint = 0;     // > 0: producer waits with try_wait suspend-time hint (ns) instead of psleep
@@ -172,6 +176,16 @@ struct Mode {
     struct Xfer { int arr, below, above; };
     std::vector<std::vector<Xfer>> xsched;
     bool xsched_ok = false;
+    // TEMP renaming and the launch DAG (options rename / streams, one rank, fused mode):
+    // per launch and array the buffer instance its HBM reads / stores use (0 = the bound
+    // buffer, k > 0 = the program's k-th shadow of that array), the launches each depends
+    // on (RAW/WAR/WAW on instances) and the stream index each is issued on
+    std::vector<std::vector<int>> rd_inst, wr_inst;
+    std::vector<int> n_inst;
+    std::vector<std::vector<int>> deps;
+    std::vector<int> stream_of;
+    bool dag_ok = false;
+    std::vector<void *> shadow_src;  // per array: the bound buffer its shadows were copied from
 };
 
 }  // namespace sf
@@ -205,6 +219,8 @@ struct stencil_program_s {
     std::vector<void *> events;  // cudaEvent_t pool for exchange overlap
     bool no_pdl = false;         // multi-rank schedule: plain stream order between launches
     std::vector<void *> wave_streams, wave_events;  // z-wave schedule: streams, events
+    std::vector<void *> dag_streams, dag_events;    // launch-DAG streams (option streams)
+    std::vector<std::vector<void *>> shadow;        // per array: renamed TEMP instances (option rename)
     std::map<int, sp_tile_config> tune_fused, tune_unfused;  // sp_plan_tune overrides
     // peer-push exchange: neighbours' buffers of each array (0 = below, 1 = above),
     // this program's signal block (u64 from_dn, from_up, self; u32 cta counter) and
@@ -250,6 +266,11 @@ double codegen_smem_loads(const Launch &L);  // shared-memory loads per core poi
 // jit.cpp
 void compile_mode(stencil_program *p, Mode &m);
 void load_mode(stencil_program *p, Mode &m);
+// TEMP instances and the launch DAG of a mode (options rename / streams); idempotent
+void dag_analysis(stencil_program *p, Mode &m, bool fused);
+// shadow buffers of renamed TEMPs: allocated and initialised from the bound buffer (ghost
+// cells) when the bindings changed, on `stream`
+void prepare_shadows(stencil_program *p, Mode &m, void *stream);
 // one launch over output planes [z0, z1) and [z2, z3) of the slab (z1 < 0: the
 // whole slab; an empty second range by default), each tiled by chunks of zc planes
 void launch(stencil_program *p, Mode &m, int i, void *stream, int z0 = 0, int z1 = -1, int z2 = 0,

@@ -38,7 +38,7 @@ def _coefs(rng, n):
     return [float(x) for x in c]
 
 
-def c4(nx=1280, ny=32, nz=256, seed=40, n_vars=5):
+def c4(nx=1280, ny=32, nz=256, seed=40, n_vars=5, reuse_temps=True):
     rng = np.random.default_rng(seed)
     # kernels are first built with symbolic temps ("d{v}_{i}", "f{v}_{i}", "tend{v}")
     ks = []
@@ -104,6 +104,13 @@ def c4(nx=1280, ny=32, nz=256, seed=40, n_vars=5):
                 for key in ("a", "b"):
                     if key in t and is_sym(t[key][0]):
                         last_read[t[key][0]] = ki
+    if not reuse_temps:  # every symbolic temp its own array (no WAR/WAW through reuse)
+        syms = []
+        for k in ks:
+            for st in k["stmts"]:
+                if is_sym(st["out"]) and st["out"] not in syms:
+                    syms.append(st["out"])
+        last_read = {n: 1 << 30 for n in syms}  # never freed
     assign, free, used = {}, list(range(64)), 0
     live = {}
     for ki, k in enumerate(ks):
@@ -119,7 +126,7 @@ def c4(nx=1280, ny=32, nz=256, seed=40, n_vars=5):
             if lr <= ki:
                 free.append(assign[n])
                 del live[n]
-    if used > 16:
+    if used > 16 and reuse_temps:
         raise RuntimeError(f"TEMP pool needs {used} > 16 arrays")
 
     def ren(n):

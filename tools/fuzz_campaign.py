@@ -48,8 +48,14 @@ def single(seed, boxes, frame=False):
     # frame shapes (free tile_y) apply to fused groups; the unfused kernels keep the block form
     uopts = {"fmad": 0} if frame else opts
     assert_close(prog, gpu_run(prog, "unfused", seed, options=uopts, poison=False), ref, exact=True)
+    from paper_conf_hpdc_wahibm15_b200 import StencilError
     for plan in plans:
-        got = gpu_run(prog, "fused", seed, options=opts, plan=plan, poison=False)
+        try:
+            got = gpu_run(prog, "fused", seed, options=opts, plan=plan, poison=False)
+        except StencilError as e:  # a pinned frame shape whose rings do not fit this group
+            if e.code == 6 and frame and "tile_x" in opts:
+                continue
+            raise
         assert_close(prog, got, ref, exact=True)
 
 

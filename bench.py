@@ -3,8 +3,9 @@
   python bench.py [--gpus N] [--steps K] [--warmup W] [--workload C4] [--impl ours|reference]
 
 One step = one pass of the whole hot path over the workload: every group of the
-fusion plan, in plan order (run_fused), plus on N > 1 ranks the z-slab halo
-exchanges.  Metric (BASELINE.json): grid-point updates/s (interior points x
+fusion plan (run_fused: on one rank along the group dependency DAG on two streams, TEMPs
+renamed per writer group; on N > 1 ranks in plan order), plus on N > 1 ranks the z-slab
+halo exchanges.  Metric (BASELINE.json): grid-point updates/s (interior points x
 original kernels / s, reading R21) and HBM GB/s against the roofline, fused vs
 unfused.  N > 1: one process per GPU (torchrun), z-slab decomposition, weak
 scaling (per-GPU grid fixed).  Inputs: seeded synthetic fields (synth/), 2.1 GB
@@ -408,6 +409,8 @@ def run_ours(args):
             "config": {"workload": args.workload, "grid_per_gpu": [prog["grid"]["nx"], prog["grid"]["ny"], nz],
                        "kernels": n_kernels, "arrays": len(prog["arrays"]),
                        "plan": args.plan, "fused_groups": len(live_f),
+                       # the fused step's launch DAG (TEMP renaming + streams, one rank)
+                       "launch_streams": (1 + max(st for _, st in p.dag("fused"))) if world == 1 else 1,
                        "parallelism": f"z-slab x{world}",
                        "halo_exchange": ("peer-push (TEMP) + NCCL (step-start)" if xpush else
                                          "NCCL send/recv") if world > 1 else "none",

@@ -236,7 +236,8 @@ sp_status stencil_program_bind(stencil_program *prog, int32_t array, void *dev_p
  *               1: a second, predicate-free copy of the step body for interior
  *               tiles/planes (fewer issued instructions, larger code); default 0
  *   "minblocks" __launch_bounds__ minimum resident CTAs (ptxas register budget)
- *   "rename"    1 (default): in run_fused on one rank, every later group that stores a
+ *   "rename"    1 (default): in run_fused on one rank of an undecomposed grid
+ *               (nz_global == nz_local), every later group that stores a
  *               TEMP array stores into its own instance (a library-allocated buffer of
  *               the program layout; extra memory = sum over TEMPs of (writer groups - 1)
  *               arrays), so TEMP reuse creates no WAR/WAW ordering between groups.  The

@@ -309,7 +309,10 @@ void dag_analysis(stencil_program *p, Mode &m, bool fused) {
     if (m.dag_ok) return;
     const int n = (int)m.launches.size(), na = (int)p->arrays.size();
     const bool multi = p->comm && p->comm->nranks > 1;
-    const bool ren = fused && p->opt.rename && !multi && p->opt.zwave == 0 && p->opt.loader == 0;
+    // a z-slab of a decomposed grid (nz_global > nz_local) exchanges ghost planes of the
+    // BOUND buffers (the library's schedule or the caller's copies): no renaming there
+    const bool slab = p->grid.nz_global != p->grid.nz_local;
+    const bool ren = fused && p->opt.rename && !multi && !slab && p->opt.zwave == 0 && p->opt.loader == 0;
     std::vector<bool> renamable(na, false);
     if (ren) {
         for (int a = 0; a < na; ++a) renamable[a] = p->arrays[a].role == SP_TEMP;

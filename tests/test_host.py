@@ -703,3 +703,31 @@ def test_ring_and_barrier_options_codegen():
     assert "sf_bar_arrive(2 + ((k - KF)" in src and "sf_bar_sync(2 + ((s - KF)" in src
     assert "sf_mbar_arrive(&empty" not in src
     b.compile("fused")
+
+
+def test_launch_dag_with_temp_renaming():
+    """sp_plan_dag: with TEMP renaming (default) C4's diag groups become roots and only the
+    real data flow orders the groups; without it every group hangs on its predecessors'
+    TEMP reuse (WAR/WAW); streams follow the latest dependency; slabs of a decomposed
+    grid and the unfused mode never rename."""
+    from synth.scale_les import c4
+    import json
+    prog = c4(nx=64, ny=32, nz=16)
+    plan = json.load(open(os.path.join(ROOT, "configs", "c4_plan.json")))["groups"]
+    p = Program(prog)
+    p.set_plan(plan)
+    dag = p.dag()
+    assert [d for d, _ in dag] == [[], [0], [], [0, 2], [], [2, 3, 4], [], [4, 6], [], [6, 8]]
+    assert {s for _, s in dag} == {0, 1}
+    for i, (d, s) in enumerate(dag):
+        if d:
+            assert s == dag[d[-1]][1]
+    q = Program(prog, options={"rename": 0, "streams": 1})
+    q.set_plan(plan)
+    dq = q.dag()
+    assert all(i == 0 or (i - 1) in d for i, (d, _) in enumerate(dq))  # a chain
+    assert {s for _, s in dq} == {0}
+    slab = Program(prog, nz_global=32, z_offset=0, zhalo=4)
+    slab.set_plan(plan)
+    assert all(i == 0 or (i - 1) in d for i, (d, _) in enumerate(slab.dag()))
+    assert all(s == 0 for _, s in p.dag("unfused"))

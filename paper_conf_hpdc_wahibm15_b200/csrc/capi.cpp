@@ -233,7 +233,10 @@ static void run_dag(stencil_program *p, Mode &m, void *stream) {
     for (int s : m.stream_of) S = std::max(S, s + 1);
     while ((int)p->dag_streams.size() < S - 1) {
         cudaStream_t s;
-        if (cudaStreamCreateWithFlags(&s, cudaStreamNonBlocking) != cudaSuccess)
+        int lo = 0, hi = 0;  // numerically: lo = least priority (0), hi = greatest (negative)
+        cudaDeviceGetStreamPriorityRange(&lo, &hi);
+        const int prio = p->opt.dagprio == 1 ? hi : p->opt.dagprio == 2 ? lo : 0;
+        if (cudaStreamCreateWithPriority(&s, cudaStreamNonBlocking, prio) != cudaSuccess)
             fail(SP_E_CUDA, "cudaStreamCreate");
         p->dag_streams.push_back(s);
     }
@@ -481,6 +484,7 @@ sp_status sp_program_set_option(stencil_program *p, const char *key, int64_t v) 
         else if (k == "pbar") o.pbar = v != 0;
         else if (k == "rename") o.rename = v != 0;
         else if (k == "streams") o.streams = (int)std::max<int64_t>(1, std::min<int64_t>(v, 8));
+        else if (k == "dagprio") o.dagprio = (int)std::min<int64_t>(v, 2);
         else if (k == "l2_flush") {}
         else fail(SP_E_ARG, "unknown option '" + k + "'");
         if (v < 0 && k != "prefetch") fail(SP_E_ARG, "negative option value");

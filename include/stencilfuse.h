@@ -246,6 +246,7 @@ sp_status stencil_program_bind(stencil_program *prog, int32_t array, void *dev_p
  *   "streams"   N (default 2): run_fused on one rank issues the launches along the group
  *               dependency DAG (sp_plan_dag) on up to N streams forked from and joined
  *               back into the caller's stream (events; graph-capturable); 1: in order
+ *   "dagprio", "dagsched"   launch-DAG stream priority / assignment variants (measured off)
  *   "psleep"    ns: the TMA producer warp waits for a free ring slot with nanosleep
  *               back-off starting at this value (default 32; 0 = spin on try_wait)
  *   "phint", "pbar", "pow2ring"   measured-off producer-wait / ring experiments

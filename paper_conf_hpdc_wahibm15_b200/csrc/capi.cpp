@@ -485,6 +485,7 @@ sp_status sp_program_set_option(stencil_program *p, const char *key, int64_t v) 
         else if (k == "rename") o.rename = v != 0;
         else if (k == "streams") o.streams = (int)std::max<int64_t>(1, std::min<int64_t>(v, 8));
         else if (k == "dagprio") o.dagprio = (int)std::min<int64_t>(v, 2);
+        else if (k == "dagsched") o.dagsched = (int)std::min<int64_t>(v, 1);
         else if (k == "l2_flush") {}
         else fail(SP_E_ARG, "unknown option '" + k + "'");
         if (v < 0 && k != "prefetch") fail(SP_E_ARG, "negative option value");

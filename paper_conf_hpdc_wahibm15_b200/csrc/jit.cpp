@@ -361,7 +361,9 @@ void dag_analysis(stencil_program *p, Mode &m, bool fused) {
     std::vector<int> load(S, 0);
     for (int i = 0; i < n; ++i) {
         int s = 0;
-        if (!m.deps[i].empty()) s = m.stream_of[m.deps[i].back()];
+        if (p->opt.dagsched == 1 && S > 1)  // roots (no dependency) run ahead on the last stream
+            s = m.deps[i].empty() ? S - 1 : 0;
+        else if (!m.deps[i].empty()) s = m.stream_of[m.deps[i].back()];
         else s = (int)(std::min_element(load.begin(), load.end()) - load.begin());
         m.stream_of[i] = s;
         load[s] += m.launches[i].dead ? 0 : 1;

@@ -58,6 +58,7 @@ struct Options {
                        // buffer instance (no WAR/WAW through TEMP reuse between groups)
     int streams = 2;   // fused mode, one rank: launches on up to this many streams along the
                        // group dependency DAG (events between streams); r2: C4 -8.3 %
+    int dagsched = 0;  // DAG stream assignment: 0 follow the latest dependency, 1 roots on their own stream
     int dagprio = 0;   // launch-DAG streams' priority: 0 default, 1 higher, 2 lower than default
     int pbar = 0;      // 1: "slot free" via named barriers (producer blocks in bar.sync, no polling)
     int pow2ring = 0;  // ring depths rounded up to powers of two (slot = mask, more shared memory)

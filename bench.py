@@ -418,6 +418,10 @@ def run_ours(args):
             **({"functional_test": "SF_BENCH_SHARE_GPU=1: all ranks share one GPU; not a measurement"}
                if os.environ.get("SF_BENCH_SHARE_GPU") == "1" else {}),
             "hbm_gbs_alg": alg_step / (step_ms * 1e-3) / 1e9,
+            # the launches one at a time in plan order (the per-launch pass) against the step,
+            # which runs them along the group DAG: what the concurrency recovers
+            "launch_dag": {"serial_launch_sum_ms": sum(per_launch[i] for i in live_f),
+                           "step_ms": step_ms},
             "roofline_step": {"achieved": alg_step / (step_ms * 1e-3) / 1e9, "peak": peak,
                               "unit": "GB/s", "frac": alg_step / (step_ms * 1e-3) / 1e9 / peak,
                               "frac_of_8tbs_nominal": alg_step / (step_ms * 1e-3) / 8e12},
